@@ -1,0 +1,409 @@
+#!/usr/bin/env python
+"""Benchmark of the MDNorm + BinMD cross-section hot path (BASELINE.json metric).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+  (N > 1: launched by torchrun, one process per GPU, NCCL)
+
+Workload (BASELINE.json configs[1], the config the metric is quoted on):
+CORELLI-shaped single run -- 372,736 pixels x 24 symmetry ops (6/mmm) = 8,945,664
+pixel-trajectories, 600x600x1 HK0 grid, 10^7 events (70% diffuse, 30% Bragg, Morton order).
+One step = mdnorm_reset + MDNorm + BinMD (+ one NCCL reduce of the packed [norm | binmd] buffer
+when N > 1) + cross-section: Algorithm 1 for one file per GPU.  Weak scaling: rank r
+processes run r of a rotation scan (omega = 17 + 3r degrees, its own seeded events), so per-GPU
+work is fixed.  value = pixel-trajectories of all ranks / max-over-ranks step time.
+
+Prints ONE JSON line on rank 0 (contract in the task statement; fields documented in DESIGN.md §6).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "MDNorm pixel-trajectories/s (full MDNorm+BinMD+xs step; BinMD events/s in 'secondary')"
+UNIT = "pixel-trajectories/s"
+
+# ----------------------------------------------------------------------------- roofline constants
+# Algorithmic fp64 operations (IEEE +,-,*,/ each counted once) per unit.
+OPS_PER_TRAJ = 24      # v = M q (9 mul + 6 add) + clip (3 x (1 div + 2 mul))
+OPS_PER_HIT = 7        # F(k_in) interpolation (6) + Omega*c (1)
+OPS_PER_SEG = 22       # crossing (3) + F(k2) (6) + midpoint (2) + 3 bin coords (9) + value (2)
+OPS_PER_PAIR = 21      # x = N q (9 mul + 6 add) + 3 x (sub, mul)
+BYTES_PER_EVENT = 16   # packed float4 (w, Qx, Qy, Qz), read once
+FP64_LANES_PER_SM = 64  # B200 FP64 pipe: 64 DADD/DMUL/DFMA per SM per clock (37 TFLOP/s FMA-counted)
+
+
+def fp64_peak_tops(sm_mhz: float, n_sm: int = 148) -> float:
+    """Peak non-fused fp64 operations/s (T): the definition forbids FMA contraction, so every
+    algorithmic + - * is one FP64-pipe instruction."""
+    return n_sm * FP64_LANES_PER_SM * sm_mhz * 1e6 / 1e12
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            return json.load(f), "measured"
+    return {"hbm_gbs": 6650.0, "sm_max_mhz": 1965.0}, "fallback"
+
+
+def ncu_traffic():
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            return json.load(f)
+    return {}
+
+
+# ----------------------------------------------------------------------------- clocks
+
+
+class ClockSampler:
+    """nvidia-smi-equivalent sampling (NVML) of SM clock and throttle reasons every 200 ms."""
+
+    def __init__(self, device_index: int):
+        self.samples, self.reasons = [], set()
+        self.max_mhz = None
+        self._stop = threading.Event()
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(device_index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.names = {
+                pynvml.nvmlClocksEventReasonGpuIdle: "gpu_idle",
+                pynvml.nvmlClocksEventReasonApplicationsClocksSetting: "applications_clocks_setting",
+                pynvml.nvmlClocksEventReasonSwPowerCap: "sw_power_cap",
+                pynvml.nvmlClocksEventReasonHwSlowdown: "hw_slowdown",
+                pynvml.nvmlClocksEventReasonSyncBoost: "sync_boost",
+                pynvml.nvmlClocksEventReasonSwThermalSlowdown: "sw_thermal_slowdown",
+                pynvml.nvmlClocksEventReasonHwThermalSlowdown: "hw_thermal_slowdown",
+                pynvml.nvmlClocksEventReasonHwPowerBrakeSlowdown: "hw_power_brake_slowdown",
+                pynvml.nvmlClocksEventReasonDisplayClockSetting: "display_clock_setting",
+            }
+        except Exception as e:  # pragma: no cover
+            self.nv = None
+            self.err = str(e)
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for bit, name in self.names.items():
+                    if r & bit:
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            self._stop.wait(0.2)
+
+    def __enter__(self):
+        if self.nv:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *exc):
+        self._stop.set()
+        if self.nv:
+            self.t.join()
+
+    def summary(self):
+        if not self.nv:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvml unavailable"]}
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
+                "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons - {"gpu_idle"}),
+                "samples": len(self.samples)}
+
+
+# ----------------------------------------------------------------------------- workload
+
+
+def make_bench_workload(world: int):
+    import synth
+    wl = synth.make_workload("corelli")
+    if world > 1:
+        wl.R = np.stack([synth.rot_y(17.0 + 3.0 * r) for r in range(world)])
+        wl.charge = np.ones(world)
+    return wl
+
+
+def config_dict(wl, world):
+    return {"workload": "corelli (BASELINE.json configs[1])", "pixels": wl.npix, "ops": wl.nops,
+            "runs_per_gpu": 1, "trajectories_per_gpu": wl.npix * wl.nops,
+            "events_per_gpu": wl.events_per_run, "grid": [int(x) for x in wl.nbins],
+            "grid_extent": [[float(a), float(b)] for a, b in zip(wl.lo, wl.hi)],
+            "event_order": "coarse-Q Morton (MDBox/SaveMD order)", "acc": "fp64",
+            "l2": "flushed between timed steps (256 MiB device write)",
+            "parallelism": f"dp{world} (rank r = run r; one NCCL reduce of [norm|binmd])" if world > 1
+            else "single GPU"}
+
+
+# ----------------------------------------------------------------------------- reference arm
+
+
+def run_reference(args, rank, world):
+    """--impl reference: the fp64 CPU oracle as it stands, on this host, per-step bounded sample."""
+    if rank != 0:
+        return 0
+    import oracle
+    import synth
+    oracle.build()
+    wl = make_bench_workload(1)
+    ev = synth.events_for_run(wl, 0)
+    stride = args.ref_stride
+    times = []
+    for k in range(args.warmup + args.steps):
+        t = {}
+        t0 = time.perf_counter()
+        oracle.run_workload(wl, events={0: ev}, pix_stride=stride, event_stride=stride, timings=t)
+        dt = time.perf_counter() - t0
+        if k >= args.warmup:
+            times.append(t["mdnorm_s"] + t["binmd_s"])
+    traj = wl.npix * wl.nops / stride
+    value = traj / statistics.mean(times)
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * statistics.mean(times),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic (seeded, SURVEY.md §8(d) recipe)", "config": config_dict(wl, 1),
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
+                             "sample": f"every {stride}th pixel (all 24 ops) and every {stride}th event "
+                                       f"of the CORELLI-shaped run per step; single-threaded C oracle"},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def cpu_baseline(wl, ev, stride):
+    import oracle
+    oracle.build()
+    t = {}
+    oracle.run_workload(wl, runs=[0], events={0: ev}, pix_stride=stride, event_stride=stride, timings=t)
+    secs = t["mdnorm_s"] + t["binmd_s"]
+    traj = wl.npix * wl.nops / stride
+    return {"value": traj / secs, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"every {stride}th pixel (all {wl.nops} ops) + every {stride}th event of run 0 "
+                      f"({traj:.0f} trajectories, {len(ev) // stride} events; "
+                      f"MDNorm {t['mdnorm_s']:.2f} s + BinMD {t['binmd_s']:.2f} s), single thread",
+            "events_per_s": (len(ev) / stride) / secs}
+
+
+# ----------------------------------------------------------------------------- our arm
+
+
+def run_ours(args, rank, world, local_rank):
+    import torch
+    import torch.distributed as dist
+    import synth
+    import paper_conf_sc_hahnfgmmshvvs24_b200 as m
+    from paper_conf_sc_hahnfgmmshvvs24_b200 import build
+
+    build.build()
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    wl = make_bench_workload(world)
+    run = rank if world > 1 else 0
+    ev = synth.events_for_run(wl, run)
+    g = m.mdnorm_create_grid(local_rank, wl.lo, wl.hi, wl.nbins, wl.W, m.MDN_ACC_F64)
+    m.mdnorm_set_instrument(g, wl.pix_dir, wl.solid)
+    m.mdnorm_set_flux(g, wl.flux_k, wl.flux_F)
+    ev_dev = torch.from_numpy(ev).to(dev)
+    packed = m.packed_histograms(g)
+    xs_dev = torch.empty(g.nbins_total, dtype=torch.float64, device=dev)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    R, c = wl.R[run], float(wl.charge[run])
+
+    def step(ph):
+        m.mdnorm_reset(g)
+        ph[0].record()
+        m.mdnorm_accumulate(g, wl.UB, R, wl.ops, wl.k_min, wl.k_max, c)
+        ph[1].record()
+        m.binmd_accumulate(g, wl.UB, wl.ops, ev_dev)
+        ph[2].record()
+        if world > 1:
+            m.reduce_packed(packed, dst=0)
+        ph[3].record()
+        if rank == 0:
+            m.mdnorm_cross_section(g, xs_dev)
+        ph[4].record()
+
+    mk = lambda: [torch.cuda.Event(enable_timing=True) for _ in range(5)]  # noqa: E731
+    # work counters from one untimed step (tracing; counted kernels are a separate variant)
+    m.mdnorm_stats(g, 1, read=False)
+    step(mk())
+    stats = m.mdnorm_stats(g, 0)
+    for _ in range(args.warmup):
+        step(mk())
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    starts = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    stops = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    phases = [mk() for _ in range(args.steps)]
+    with ClockSampler(local_rank) as clk:
+        for k in range(args.steps):
+            flush.zero_()  # L2 flush (outside the timed events)
+            starts[k].record()
+            step(phases[k])
+            stops[k].record()
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    step_ms = [a.elapsed_time(b) for a, b in zip(starts, stops)]
+    total_ms = torch.tensor([sum(step_ms)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(total_ms, op=dist.ReduceOp.MAX)
+    total_ms = float(total_ms.item())
+    ph_ms = {name: statistics.mean(p[i].elapsed_time(p[i + 1]) for p in phases)
+             for i, name in enumerate(["mdnorm", "binmd", "reduce", "xs"])}
+
+    # ---------------- end to end through the C ABI with HOST buffers (pinned), copies inside
+    ev_pin = torch.from_numpy(ev).pin_memory()
+    xs_pin = torch.empty(g.nbins_total, dtype=torch.float64).pin_memory()
+
+    def step_e2e():
+        m.mdnorm_reset(g)
+        m.mdnorm_accumulate(g, wl.UB, R, wl.ops, wl.k_min, wl.k_max, c)
+        m.binmd_accumulate(g, wl.UB, wl.ops, ev_pin)          # chunked H2D overlapped with scatter
+        if world > 1:
+            m.reduce_packed(packed, dst=0)
+        if rank == 0:
+            m.mdnorm_cross_section(g, xs_pin)                   # D2H + synchronise
+
+    for _ in range(2):
+        step_e2e()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    e_starts = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    e_stops = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    with ClockSampler(local_rank) as clk_e2e:
+        for k in range(args.steps):
+            flush.zero_()
+            e_starts[k].record()
+            step_e2e()
+            e_stops[k].record()
+        torch.cuda.synchronize()
+    e2e_ms = torch.tensor([sum(a.elapsed_time(b) for a, b in zip(e_starts, e_stops))], dtype=torch.float64,
+                          device=dev)
+    if world > 1:
+        dist.all_reduce(e2e_ms, op=dist.ReduceOp.MAX)
+    e2e_ms = float(e2e_ms.item())
+
+    # sanity: the result of the last step is a real cross-section
+    if rank == 0:
+        xs_np = xs_pin.numpy()
+        finite = np.isfinite(xs_np)
+        assert finite.sum() > 1000, "cross-section has too few finite bins"
+
+    traj_total = wl.npix * wl.nops * world
+    ev_total = len(ev) * world
+    ms_per_step = total_ms / args.steps
+    value = traj_total / (ms_per_step / 1e3)
+
+    peaks, peaks_src = measured_peaks()
+    clocks = clk.summary()
+    sm_max = float(peaks.get("sm_max_mhz", 1965.0))
+    fp64_peak = fp64_peak_tops(sm_max)
+    hbm = float(peaks["hbm_gbs"])
+    traffic = ncu_traffic()
+    kernels = {}
+    md_ops = OPS_PER_TRAJ * stats["trajectories"] + OPS_PER_HIT * stats["hit_trajectories"] + \
+        OPS_PER_SEG * stats["segments"]
+    t = ph_ms["mdnorm"] / 1e3
+    kernels["mdnorm_kernel"] = {"bound": "alu", "achieved": md_ops / t / 1e12, "peak": fp64_peak,
+                                "unit": "TFLOP/s", "frac": md_ops / t / 1e12 / fp64_peak,
+                                "traffic": traffic.get("mdnorm_kernel"), "ms": ph_ms["mdnorm"],
+                                "ops_per_launch": md_ops,
+                                "peak_note": f"fp64 non-fused ops at {sm_max:.0f} MHz (148 SM x 64 lanes), "
+                                             "DESIGN.md §4"}
+    t = ph_ms["binmd"] / 1e3
+    bm_bytes = BYTES_PER_EVENT * len(ev)
+    bm_ops = OPS_PER_PAIR * stats["event_op_pairs"]
+    kernels["binmd_kernel"] = {"bound": "alu", "achieved": bm_ops / t / 1e12, "peak": fp64_peak,
+                               "unit": "TFLOP/s", "frac": bm_ops / t / 1e12 / fp64_peak,
+                               "traffic": traffic.get("binmd_kernel"), "ms": ph_ms["binmd"],
+                               "hbm_gbs": bm_bytes / t / 1e9, "hbm_frac": bm_bytes / t / 1e9 / hbm}
+    t = ph_ms["xs"] / 1e3
+    if rank == 0 and t > 0:
+        xs_bytes = 24 * g.nbins_total
+        kernels["xs_kernel"] = {"bound": "hbm", "achieved": xs_bytes / t / 1e9, "peak": hbm, "unit": "GB/s",
+                                "frac": xs_bytes / t / 1e9 / hbm, "ms": ph_ms["xs"]}
+    dom = max(("mdnorm_kernel", "binmd_kernel"), key=lambda k: kernels[k]["ms"])
+    roof = {k: kernels[dom][k] for k in ("bound", "achieved", "peak", "unit", "frac", "traffic")}
+    roof["kernel"] = dom
+    roof["peak_source"] = f"{peaks_src} (MEASURED_PEAKS.json sm_max_mhz; fp64 lanes from the B200 spec)"
+
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f64", "data": "synthetic (seeded, SURVEY.md §8(d) CORELLI recipe)",
+        "config": config_dict(wl, world),
+        "secondary": {"binmd_events_per_s": ev_total / (ms_per_step / 1e3),
+                      "mdnorm_kernel_traj_per_s": wl.npix * wl.nops / (ph_ms["mdnorm"] / 1e3),
+                      "binmd_kernel_events_per_s": len(ev) / (ph_ms["binmd"] / 1e3),
+                      "mdnorm_segments_per_s": stats["segments"] / (ph_ms["mdnorm"] / 1e3),
+                      "phase_ms": ph_ms, "work_counts_rank0": stats},
+        "clocks": clocks,
+        "e2e": {"value": traj_total / (e2e_ms / args.steps / 1e3), "unit": UNIT,
+                "ms_per_step": e2e_ms / args.steps,
+                "h2d_bytes_per_step": int(ev.nbytes) * world,
+                "d2h_bytes_per_step": 8 * g.nbins_total,
+                "clocks": clk_e2e.summary(),
+                "path": "C ABI with pinned host events (chunked H2D overlapped with BinMD) and host xs"},
+        "gpu_launches": args.steps * (2 + (1 if rank == 0 else 0)),
+        "roofline": roof,
+        "kernels": kernels,
+    }
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        line["cpu_baseline"] = cpu_baseline(wl, ev, args.cpu_stride)
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+        if args.json_out:
+            with open(args.json_out, "w") as f:
+                json.dump(line, f, indent=1)
+    g.close()
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-stride", type=int, default=2, help="oracle sample: every n-th pixel and event")
+    ap.add_argument("--ref-stride", type=int, default=8, help="--impl reference per-step sample stride")
+    ap.add_argument("--json-out", default=None)
+    args = ap.parse_args()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        return run_reference(args, rank, world)
+    if world > 1:
+        import torch
+        import torch.distributed as dist
+        torch.cuda.set_device(local_rank)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    try:
+        return run_ours(args, rank, world, local_rank)
+    finally:
+        if world > 1:
+            import torch.distributed as dist
+            dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    sys.exit(main())

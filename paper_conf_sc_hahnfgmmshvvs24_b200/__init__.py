@@ -1,0 +1,14 @@
+"""B200-native MDNorm + BinMD single-crystal TOF cross-section hot path (Hahn et al., SC'24 W).
+
+The product is the C-ABI library libmdnorm.so (include/mdnorm.h); this package is its thin
+Python binding (same function names) plus the multi-GPU shard plan / reduce (dist.py).
+"""
+from .mdnorm import (  # noqa: F401
+    Grid, MdnError, MDN_ACC_F32, MDN_ACC_F64,
+    mdnorm_create_grid, mdnorm_destroy, mdnorm_set_instrument, mdnorm_set_flux,
+    mdnorm_accumulate, mdnorm_accumulate_runs, binmd_accumulate, mdnorm_histograms,
+    mdnorm_cross_section, mdnorm_reset, mdnorm_stats, mdn_last_error, mdn_version,
+    mdnorm_accumulate_matrices, binmd_accumulate_matrices, mdnorm_debug_trajectories,
+    binmd_debug_bins, mdnorm_debug_compose, packed_histograms,
+)
+from .dist import plan_shards, reduce_packed, RankPlan  # noqa: F401

@@ -1,0 +1,660 @@
+// mdn_api.cu -- the extern "C" boundary declared in include/mdnorm.h.
+//
+// Host side only: argument validation (before any side effect), device-memory ownership,
+// stream ordering and launch marshalling.  Every step of the hot path itself (matrix
+// composition, trajectories, scatter, divide) runs in the kernels of mdn_kernels.cu.
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "mdn_kernels.cuh"
+#include "mdnorm.h"
+
+using mdn::GridC;
+using mdn::MatBlock;
+
+struct mdn_grid {
+  int device = 0;
+  int num_sms = 148;
+  GridC g{};
+  double W[9]{};
+  mdn_acc acc = MDN_ACC_F64;
+  double* d_hist = nullptr;  // [norm | binmd], 2 * nbins doubles
+  double4* d_pix = nullptr;
+  int64_t npix = 0;
+  double* d_flux = nullptr;  // [k | F], 2 * nflux doubles
+  int32_t nflux = 0;
+  double* d_xs = nullptr;    // scratch for host xs
+  unsigned long long* d_stats = nullptr;  // 6 work counters (mdnorm_stats)
+  bool stats_on = false;
+  // host-event streaming (binmd_accumulate with a host pointer)
+  float* d_stage[2] = {nullptr, nullptr};
+  size_t stage_floats = 0;
+  cudaStream_t copy_stream = nullptr;
+  cudaEvent_t ev_ready[2] = {nullptr, nullptr};
+  cudaEvent_t ev_free[2] = {nullptr, nullptr};
+};
+
+namespace {
+
+thread_local std::string g_err;
+
+mdn_status fail(mdn_status st, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  g_err = buf;
+  return st;
+}
+
+mdn_status cuda_fail(cudaError_t e, const char* where) {
+  cudaGetLastError();  // clear sticky-free errors
+  return fail(e == cudaErrorMemoryAllocation ? MDN_ENOMEM : MDN_ECUDA, "%s: %s", where,
+              cudaGetErrorString(e));
+}
+
+#define MDN_CUDA(call, where)                   \
+  do {                                          \
+    cudaError_t e_ = (call);                    \
+    if (e_ != cudaSuccess) return cuda_fail(e_, where); \
+  } while (0)
+
+mdn_status ok() {
+  g_err.clear();
+  return MDN_OK;
+}
+
+// Restores the caller's current device on scope exit.
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur;
+    if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+bool finite_all(const double* x, int64_t n) {
+  for (int64_t i = 0; i < n; ++i)
+    if (!std::isfinite(x[i])) return false;
+  return true;
+}
+
+double det3(const double* m) {
+  return m[0] * (m[4] * m[8] - m[5] * m[7]) - m[1] * (m[3] * m[8] - m[5] * m[6]) +
+         m[2] * (m[3] * m[7] - m[4] * m[6]);
+}
+
+bool nonsingular(const double* m) {
+  double d = det3(m);
+  return std::isfinite(d) && d != 0.0;
+}
+
+bool is_device_ptr(const void* p) {
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+// copy n elements from a host or device pointer into a host vector
+template <class T>
+cudaError_t to_host(const T* src, int64_t n, std::vector<T>& dst) {
+  dst.resize((size_t)n);
+  if (n == 0) return cudaSuccess;
+  if (is_device_ptr(src)) return cudaMemcpy(dst.data(), src, sizeof(T) * n, cudaMemcpyDeviceToHost);
+  std::memcpy(dst.data(), src, sizeof(T) * n);
+  return cudaSuccess;
+}
+
+mdn_status check_ops(int32_t nops, const double* ops) {
+  if (nops < 1 || nops > MDN_MAX_OPS) return fail(MDN_EINVAL, "nops = %d outside [1, %d]", nops, MDN_MAX_OPS);
+  if (!ops) return fail(MDN_EINVAL, "ops is NULL");
+  if (!finite_all(ops, 9 * (int64_t)nops)) return fail(MDN_EINVAL, "ops contain non-finite values");
+  for (int s = 0; s < nops; ++s)
+    if (!nonsingular(ops + 9 * s)) return fail(MDN_EINVAL, "symmetry op %d is singular", s);
+  return MDN_OK;
+}
+
+mdn_status check_matrix(const double* m, const char* name) {
+  if (!m) return fail(MDN_EINVAL, "%s is NULL", name);
+  if (!finite_all(m, 9)) return fail(MDN_EINVAL, "%s has non-finite values", name);
+  if (!nonsingular(m)) return fail(MDN_EINVAL, "%s is singular", name);
+  return MDN_OK;
+}
+
+mdn_status check_krange(double k_min, double k_max) {
+  if (!(std::isfinite(k_min) && std::isfinite(k_max) && k_min > 0.0 && k_min < k_max))
+    return fail(MDN_EINVAL, "need 0 < k_min < k_max (got %g, %g)", k_min, k_max);
+  return MDN_OK;
+}
+
+mdn_status check_ready(mdn_grid* g) {
+  if (!g) return fail(MDN_EINVAL, "grid is NULL");
+  if (!g->d_pix) return fail(MDN_ESTATE, "mdnorm_set_instrument has not been called");
+  if (!g->d_flux) return fail(MDN_ESTATE, "mdnorm_set_flux has not been called");
+  return MDN_OK;
+}
+
+mdn_status shard(mdn_grid* g, int64_t pix_begin, int64_t pix_end, int64_t pix_stride, int64_t* nshard) {
+  if (pix_end < 0) pix_end = g->npix;
+  if (pix_begin < 0 || pix_end > g->npix || pix_stride < 1)
+    return fail(MDN_EINVAL, "bad pixel shard [%lld, %lld) stride %lld for npix %lld", (long long)pix_begin,
+                (long long)pix_end, (long long)pix_stride, (long long)g->npix);
+  *nshard = pix_begin < pix_end ? (pix_end - pix_begin + pix_stride - 1) / pix_stride : 0;
+  return MDN_OK;
+}
+
+mdn::MdnParams mdn_params(mdn_grid* g, double k_min, double k_max, int64_t pix_begin, int64_t pix_stride,
+                          int64_t nshard) {
+  mdn::MdnParams p{};
+  p.g = g->g;
+  p.pix = g->d_pix;
+  p.pix_begin = pix_begin;
+  p.pix_stride = pix_stride;
+  p.nshard = nshard;
+  p.flux_k = g->d_flux;
+  p.flux_F = g->d_flux + g->nflux;
+  p.nflux = g->nflux;
+  p.acc_f32 = g->acc == MDN_ACC_F32;
+  p.kmin = k_min;
+  p.kmax = k_max;
+  p.norm = g->d_hist;
+  p.stats = g->stats_on ? g->d_stats : nullptr;
+  return p;
+}
+
+mdn_status check_events(int64_t nevents, const float* events, int64_t stride, int32_t col_w, int32_t col_q) {
+  if (nevents < 0) return fail(MDN_EINVAL, "nevents < 0");
+  if (nevents > 0 && !events) return fail(MDN_EINVAL, "events is NULL");
+  if (stride < 4 || col_w < 0 || col_q < 0 || col_w >= stride || col_q + 3 > stride ||
+      (col_w >= col_q && col_w < col_q + 3))
+    return fail(MDN_EINVAL, "bad event layout: stride %lld, col_w %d, col_q %d", (long long)stride, col_w, col_q);
+  return MDN_OK;
+}
+
+mdn::BinParams bin_params(mdn_grid* g, const float* ev, int64_t n, int64_t stride, int32_t col_w, int32_t col_q) {
+  mdn::BinParams p{};
+  p.g = g->g;
+  p.events = ev;
+  p.nevents = n;
+  p.stride = stride;
+  p.col_w = col_w;
+  p.col_q = col_q;
+  p.acc_f32 = g->acc == MDN_ACC_F32;
+  p.binmd = g->d_hist + g->g.nbins;
+  p.stats = g->stats_on ? g->d_stats : nullptr;
+  return p;
+}
+
+// Run the BinMD kernel over host events through a two-slot staging ring: the H2D copy of chunk
+// c+1 (copy stream) overlaps the scatter of chunk c (caller's stream).
+mdn_status binmd_host_stream(mdn_grid* g, const MatBlock& mb, int64_t nevents, const float* events,
+                             int64_t stride, int32_t col_w, int32_t col_q, cudaStream_t s) {
+  const int64_t chunk = std::max<int64_t>(1, (int64_t)(64ll << 20) / (int64_t)(4 * stride));  // 64 MB
+  const size_t need = (size_t)(chunk * stride);
+  if (g->stage_floats < need) {
+    for (int i = 0; i < 2; ++i) {
+      if (g->d_stage[i]) cudaFree(g->d_stage[i]);
+      g->d_stage[i] = nullptr;
+    }
+    g->stage_floats = 0;
+    for (int i = 0; i < 2; ++i) MDN_CUDA(cudaMalloc(&g->d_stage[i], need * sizeof(float)), "staging alloc");
+    g->stage_floats = need;
+  }
+  if (!g->copy_stream) {
+    MDN_CUDA(cudaStreamCreateWithFlags(&g->copy_stream, cudaStreamNonBlocking), "copy stream");
+    for (int i = 0; i < 2; ++i) {
+      MDN_CUDA(cudaEventCreateWithFlags(&g->ev_ready[i], cudaEventDisableTiming), "event");
+      MDN_CUDA(cudaEventCreateWithFlags(&g->ev_free[i], cudaEventDisableTiming), "event");
+    }
+  }
+  // the first copy may not run ahead of earlier work on the caller's stream that uses staging
+  for (int i = 0; i < 2; ++i) {
+    MDN_CUDA(cudaEventRecord(g->ev_free[i], s), "event record");
+  }
+  int64_t c = 0;
+  for (int64_t off = 0; off < nevents; off += chunk, ++c) {
+    const int slot = (int)(c & 1);
+    const int64_t n = std::min(chunk, nevents - off);
+    MDN_CUDA(cudaStreamWaitEvent(g->copy_stream, g->ev_free[slot], 0), "wait");
+    MDN_CUDA(cudaMemcpyAsync(g->d_stage[slot], events + off * stride, sizeof(float) * n * stride,
+                             cudaMemcpyHostToDevice, g->copy_stream), "H2D events");
+    MDN_CUDA(cudaEventRecord(g->ev_ready[slot], g->copy_stream), "event record");
+    MDN_CUDA(cudaStreamWaitEvent(s, g->ev_ready[slot], 0), "wait");
+    MDN_CUDA(mdn::launch_binmd(bin_params(g, g->d_stage[slot], n, stride, col_w, col_q), mb, g->num_sms, s),
+             "binmd kernel");
+    MDN_CUDA(cudaEventRecord(g->ev_free[slot], s), "event record");
+  }
+  return MDN_OK;
+}
+
+mdn_status binmd_run(mdn_grid* g, const MatBlock& mb, int64_t nevents, const float* events, int64_t stride,
+                     int32_t col_w, int32_t col_q, cudaStream_t s) {
+  if (nevents == 0) return ok();
+  if (is_device_ptr(events)) {
+    MDN_CUDA(mdn::launch_binmd(bin_params(g, events, nevents, stride, col_w, col_q), mb, g->num_sms, s),
+             "binmd kernel");
+    return ok();
+  }
+  mdn_status st = binmd_host_stream(g, mb, nevents, events, stride, col_w, col_q, s);
+  return st == MDN_OK ? ok() : st;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* mdn_last_error(void) { return g_err.c_str(); }
+
+const char* mdn_version(void) { return "mdnorm sm_100a 0.1.0"; }
+
+mdn_status mdnorm_create_grid(int device, const double lo[3], const double hi[3], const int64_t nbins[3],
+                              const double W[9], mdn_acc acc, mdn_grid** out) {
+  if (!out) return fail(MDN_EINVAL, "out is NULL");
+  *out = nullptr;
+  if (!lo || !hi || !nbins || !W) return fail(MDN_EINVAL, "NULL argument");
+  int64_t total = 1;
+  for (int a = 0; a < 3; ++a) {
+    if (!(std::isfinite(lo[a]) && std::isfinite(hi[a]) && lo[a] < hi[a]))
+      return fail(MDN_EINVAL, "axis %d: need finite lo < hi (got %g, %g)", a, lo[a], hi[a]);
+    if (nbins[a] < 1 || nbins[a] > (1ll << 30)) return fail(MDN_EINVAL, "axis %d: nbins %lld outside [1, 2^30]", a, (long long)nbins[a]);
+    total *= nbins[a];
+    if (total > (1ll << 40)) return fail(MDN_EINVAL, "grid too large");
+  }
+  if (!finite_all(W, 9) || !nonsingular(W)) return fail(MDN_EINVAL, "W is singular or non-finite");
+  if (acc != MDN_ACC_F64 && acc != MDN_ACC_F32) return fail(MDN_EINVAL, "unknown accumulation mode %d", (int)acc);
+  if (acc == MDN_ACC_F32) return fail(MDN_EINVAL, "MDN_ACC_F32 is not available in this build (use MDN_ACC_F64)");
+  int ndev = 0;
+  cudaError_t e = cudaGetDeviceCount(&ndev);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaGetDeviceCount");
+  if (device < 0 || device >= ndev) return fail(MDN_EINVAL, "device %d outside [0, %d)", device, ndev);
+  DeviceGuard dg(device);
+  mdn_grid* g = new mdn_grid;
+  g->device = device;
+  g->acc = acc;
+  cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, device);
+  for (int a = 0; a < 3; ++a) {
+    g->g.lo[a] = lo[a];
+    g->g.hi[a] = hi[a];
+    g->g.n[a] = (int32_t)nbins[a];
+    g->g.w[a] = (hi[a] - lo[a]) / (double)nbins[a];  // IEEE double, same as the device would
+    g->g.s[a] = 1.0 / g->g.w[a];
+  }
+  g->g.nbins = total;
+  std::memcpy(g->W, W, sizeof g->W);
+  e = cudaMalloc(&g->d_hist, sizeof(double) * 2 * (size_t)total);
+  if (e == cudaSuccess) e = cudaMemset(g->d_hist, 0, sizeof(double) * 2 * (size_t)total);
+  if (e != cudaSuccess) {
+    if (g->d_hist) cudaFree(g->d_hist);
+    delete g;
+    return cuda_fail(e, "histogram allocation");
+  }
+  *out = g;
+  return ok();
+}
+
+mdn_status mdnorm_destroy(mdn_grid* g) {
+  if (!g) return ok();
+  DeviceGuard dg(g->device);
+  cudaDeviceSynchronize();
+  cudaFree(g->d_hist);
+  cudaFree(g->d_pix);
+  cudaFree(g->d_flux);
+  cudaFree(g->d_xs);
+  cudaFree(g->d_stats);
+  for (int i = 0; i < 2; ++i) {
+    cudaFree(g->d_stage[i]);
+    if (g->ev_ready[i]) cudaEventDestroy(g->ev_ready[i]);
+    if (g->ev_free[i]) cudaEventDestroy(g->ev_free[i]);
+  }
+  if (g->copy_stream) cudaStreamDestroy(g->copy_stream);
+  delete g;
+  cudaGetLastError();
+  return ok();
+}
+
+mdn_status mdnorm_set_instrument(mdn_grid* g, int64_t npix, const double* dir, const double* solid) {
+  if (!g) return fail(MDN_EINVAL, "grid is NULL");
+  if (npix < 1 || !dir || !solid) return fail(MDN_EINVAL, "need npix >= 1 and non-NULL dir, solid");
+  DeviceGuard dg(g->device);
+  std::vector<double> hd, hs;
+  MDN_CUDA(to_host(dir, 3 * npix, hd), "read dir");
+  MDN_CUDA(to_host(solid, npix, hs), "read solid");
+  if (!finite_all(hd.data(), 3 * npix)) return fail(MDN_EINVAL, "dir has non-finite values");
+  for (int64_t i = 0; i < npix; ++i)
+    if (!(std::isfinite(hs[i]) && hs[i] >= 0.0)) return fail(MDN_EINVAL, "solid[%lld] = %g is not >= 0", (long long)i, hs[i]);
+  double *d_dir = nullptr, *d_sol = nullptr;
+  double4* d_pix = nullptr;
+  cudaError_t e = cudaMalloc(&d_pix, sizeof(double4) * npix);
+  if (e == cudaSuccess) e = cudaMalloc(&d_dir, sizeof(double) * 3 * npix);
+  if (e == cudaSuccess) e = cudaMalloc(&d_sol, sizeof(double) * npix);
+  if (e == cudaSuccess) e = cudaMemcpy(d_dir, hd.data(), sizeof(double) * 3 * npix, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemcpy(d_sol, hs.data(), sizeof(double) * npix, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = mdn::launch_pixels_prepare(d_dir, d_sol, d_pix, npix, nullptr);
+  if (e == cudaSuccess) e = cudaDeviceSynchronize();
+  cudaFree(d_dir);
+  cudaFree(d_sol);
+  if (e != cudaSuccess) {
+    cudaFree(d_pix);
+    return cuda_fail(e, "set_instrument");
+  }
+  cudaFree(g->d_pix);
+  g->d_pix = d_pix;
+  g->npix = npix;
+  return ok();
+}
+
+mdn_status mdnorm_set_flux(mdn_grid* g, int64_t n, const double* k, const double* F) {
+  if (!g) return fail(MDN_EINVAL, "grid is NULL");
+  if (n < 2 || n > (1 << 30) || !k || !F) return fail(MDN_EINVAL, "need n >= 2 and non-NULL k, F");
+  DeviceGuard dg(g->device);
+  std::vector<double> hk, hF;
+  MDN_CUDA(to_host(k, n, hk), "read k");
+  MDN_CUDA(to_host(F, n, hF), "read F");
+  if (!finite_all(hk.data(), n) || !finite_all(hF.data(), n)) return fail(MDN_EINVAL, "flux table has non-finite values");
+  for (int64_t i = 1; i < n; ++i) {
+    if (!(hk[i] > hk[i - 1])) return fail(MDN_EINVAL, "flux k not strictly increasing at %lld", (long long)i);
+    if (hF[i] < hF[i - 1]) return fail(MDN_EINVAL, "cumulative flux F decreases at %lld", (long long)i);
+  }
+  double* d = nullptr;
+  cudaError_t e = cudaMalloc(&d, sizeof(double) * 2 * n);
+  if (e == cudaSuccess) e = cudaMemcpy(d, hk.data(), sizeof(double) * n, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemcpy(d + n, hF.data(), sizeof(double) * n, cudaMemcpyHostToDevice);
+  if (e != cudaSuccess) {
+    cudaFree(d);
+    return cuda_fail(e, "set_flux");
+  }
+  cudaDeviceSynchronize();
+  cudaFree(g->d_flux);
+  g->d_flux = d;
+  g->nflux = (int32_t)n;
+  return ok();
+}
+
+mdn_status mdnorm_accumulate_runs(mdn_grid* g, const double UB[9], int32_t nruns, const double* R,
+                                  const double* charge, int32_t nops, const double* ops, double k_min,
+                                  double k_max, int64_t pix_begin, int64_t pix_end, int64_t pix_stride,
+                                  void* stream) {
+  mdn_status st;
+  if ((st = check_ready(g)) != MDN_OK) return st;
+  if ((st = check_matrix(UB, "UB")) != MDN_OK) return st;
+  if ((st = check_ops(nops, ops)) != MDN_OK) return st;
+  if ((st = check_krange(k_min, k_max)) != MDN_OK) return st;
+  if (nruns < 0 || (nruns > 0 && (!R || !charge))) return fail(MDN_EINVAL, "bad runs (nruns %d)", nruns);
+  for (int r = 0; r < nruns; ++r) {
+    if ((st = check_matrix(R + 9 * r, "R")) != MDN_OK) return st;
+    if (!(std::isfinite(charge[r]) && charge[r] >= 0.0)) return fail(MDN_EINVAL, "charge[%d] = %g is not >= 0", r, charge[r]);
+  }
+  int64_t nshard;
+  if ((st = shard(g, pix_begin, pix_end, pix_stride, &nshard)) != MDN_OK) return st;
+  DeviceGuard dg(g->device);
+  cudaStream_t s = (cudaStream_t)stream;
+  const mdn::MdnParams p = mdn_params(g, k_min, k_max, pix_begin, pix_stride, nshard);
+  const int per_launch = std::max(1, std::min(mdn::kRunsPerLaunch, 384 / nops));
+  for (int r0 = 0; r0 < nruns; r0 += per_launch) {
+    const int nr = std::min(per_launch, nruns - r0);
+    MatBlock mb{};
+    mb.compose = 1;
+    mb.nops = nops;
+    mb.nruns = nr;
+    mb.nmat = nr * nops;
+    std::memcpy(mb.UB, UB, sizeof mb.UB);
+    std::memcpy(mb.W, g->W, sizeof mb.W);
+    std::memcpy(mb.u.c.ops, ops, sizeof(double) * 9 * nops);
+    std::memcpy(mb.u.c.R, R + 9 * r0, sizeof(double) * 9 * nr);
+    std::memcpy(mb.charge, charge + r0, sizeof(double) * nr);
+    MDN_CUDA(mdn::launch_mdnorm(p, mb, g->num_sms, s), "mdnorm kernel");
+  }
+  return ok();
+}
+
+mdn_status mdnorm_accumulate(mdn_grid* g, const double UB[9], const double R[9], int32_t nops, const double* ops,
+                             double k_min, double k_max, double proton_charge, int64_t pix_begin, int64_t pix_end,
+                             int64_t pix_stride, void* stream) {
+  return mdnorm_accumulate_runs(g, UB, 1, R, &proton_charge, nops, ops, k_min, k_max, pix_begin, pix_end,
+                                pix_stride, stream);
+}
+
+mdn_status binmd_accumulate(mdn_grid* g, const double UB[9], int32_t nops, const double* ops, int64_t nevents,
+                            const float* events, int64_t stride_floats, int32_t col_w, int32_t col_q, void* stream) {
+  if (!g) return fail(MDN_EINVAL, "grid is NULL");
+  mdn_status st;
+  if ((st = check_matrix(UB, "UB")) != MDN_OK) return st;
+  if ((st = check_ops(nops, ops)) != MDN_OK) return st;
+  if ((st = check_events(nevents, events, stride_floats, col_w, col_q)) != MDN_OK) return st;
+  DeviceGuard dg(g->device);
+  MatBlock mb{};
+  mb.compose = 1;
+  mb.nops = nops;
+  mb.nmat = nops;
+  std::memcpy(mb.UB, UB, sizeof mb.UB);
+  std::memcpy(mb.W, g->W, sizeof mb.W);
+  std::memcpy(mb.u.c.ops, ops, sizeof(double) * 9 * nops);
+  return binmd_run(g, mb, nevents, events, stride_floats, col_w, col_q, (cudaStream_t)stream);
+}
+
+mdn_status mdnorm_histograms(mdn_grid* g, void** norm_dev, void** binmd_dev, int64_t* nbins_total) {
+  if (!g) return fail(MDN_EINVAL, "grid is NULL");
+  if (norm_dev) *norm_dev = g->d_hist;
+  if (binmd_dev) *binmd_dev = g->d_hist + g->g.nbins;
+  if (nbins_total) *nbins_total = g->g.nbins;
+  return ok();
+}
+
+mdn_status mdnorm_cross_section(mdn_grid* g, double* xs, void* stream) {
+  if (!g) return fail(MDN_EINVAL, "grid is NULL");
+  if (!xs) return fail(MDN_EINVAL, "xs is NULL");
+  DeviceGuard dg(g->device);
+  cudaStream_t s = (cudaStream_t)stream;
+  const int64_t n = g->g.nbins;
+  if (is_device_ptr(xs)) {
+    MDN_CUDA(mdn::launch_cross_section(g->d_hist, g->d_hist + n, xs, n, g->num_sms, s), "xs kernel");
+    return ok();
+  }
+  if (!g->d_xs) MDN_CUDA(cudaMalloc(&g->d_xs, sizeof(double) * n), "xs scratch");
+  MDN_CUDA(mdn::launch_cross_section(g->d_hist, g->d_hist + n, g->d_xs, n, g->num_sms, s), "xs kernel");
+  MDN_CUDA(cudaMemcpyAsync(xs, g->d_xs, sizeof(double) * n, cudaMemcpyDeviceToHost, s), "D2H xs");
+  MDN_CUDA(cudaStreamSynchronize(s), "sync");
+  return ok();
+}
+
+mdn_status mdnorm_reset(mdn_grid* g, void* stream) {
+  if (!g) return fail(MDN_EINVAL, "grid is NULL");
+  DeviceGuard dg(g->device);
+  MDN_CUDA(cudaMemsetAsync(g->d_hist, 0, sizeof(double) * 2 * g->g.nbins, (cudaStream_t)stream), "memset");
+  if (g->d_stats) MDN_CUDA(cudaMemsetAsync(g->d_stats, 0, sizeof(unsigned long long) * 6, (cudaStream_t)stream), "memset");
+  return ok();
+}
+
+mdn_status mdnorm_stats(mdn_grid* g, int enable, int64_t out[6]) {
+  if (!g) return fail(MDN_EINVAL, "grid is NULL");
+  if (enable < -1 || enable > 1) return fail(MDN_EINVAL, "enable must be -1, 0 or 1");
+  DeviceGuard dg(g->device);
+  if (!g->d_stats) {
+    MDN_CUDA(cudaMalloc(&g->d_stats, sizeof(unsigned long long) * 6), "stats alloc");
+    MDN_CUDA(cudaMemset(g->d_stats, 0, sizeof(unsigned long long) * 6), "stats memset");
+  }
+  if (enable >= 0) g->stats_on = enable == 1;
+  if (out) {
+    unsigned long long h[6];
+    MDN_CUDA(cudaDeviceSynchronize(), "sync");
+    MDN_CUDA(cudaMemcpy(h, g->d_stats, sizeof h, cudaMemcpyDeviceToHost), "stats D2H");
+    for (int i = 0; i < 6; ++i) out[i] = (int64_t)h[i];
+  }
+  return ok();
+}
+
+// ------------------------------------------------------------------ parity / test entry points
+
+mdn_status mdnorm_accumulate_matrices(mdn_grid* g, int32_t nmat, const double* M, const double* charge,
+                                      double k_min, double k_max, int64_t pix_begin, int64_t pix_end,
+                                      int64_t pix_stride, void* stream) {
+  mdn_status st;
+  if ((st = check_ready(g)) != MDN_OK) return st;
+  if (nmat < 1 || nmat > MDN_MAX_MATS || !M || !charge) return fail(MDN_EINVAL, "nmat %d outside [1, %d]", nmat, MDN_MAX_MATS);
+  if (!finite_all(M, 9 * (int64_t)nmat) || !finite_all(charge, nmat)) return fail(MDN_EINVAL, "non-finite matrices");
+  for (int m = 0; m < nmat; ++m)
+    if (charge[m] < 0) return fail(MDN_EINVAL, "charge[%d] < 0", m);
+  if ((st = check_krange(k_min, k_max)) != MDN_OK) return st;
+  int64_t nshard;
+  if ((st = shard(g, pix_begin, pix_end, pix_stride, &nshard)) != MDN_OK) return st;
+  DeviceGuard dg(g->device);
+  MatBlock mb{};
+  mb.compose = 0;
+  mb.nmat = nmat;
+  std::memcpy(mb.u.M, M, sizeof(double) * 9 * nmat);
+  std::memcpy(mb.charge, charge, sizeof(double) * nmat);
+  MDN_CUDA(mdn::launch_mdnorm(mdn_params(g, k_min, k_max, pix_begin, pix_stride, nshard), mb, g->num_sms,
+                              (cudaStream_t)stream), "mdnorm kernel");
+  return ok();
+}
+
+mdn_status binmd_accumulate_matrices(mdn_grid* g, int32_t nmat, const double* N, int64_t nevents, const float* events,
+                                     int64_t stride_floats, int32_t col_w, int32_t col_q, void* stream) {
+  if (!g) return fail(MDN_EINVAL, "grid is NULL");
+  if (nmat < 1 || nmat > MDN_MAX_MATS || !N) return fail(MDN_EINVAL, "nmat %d outside [1, %d]", nmat, MDN_MAX_MATS);
+  if (!finite_all(N, 9 * (int64_t)nmat)) return fail(MDN_EINVAL, "non-finite matrices");
+  mdn_status st;
+  if ((st = check_events(nevents, events, stride_floats, col_w, col_q)) != MDN_OK) return st;
+  DeviceGuard dg(g->device);
+  MatBlock mb{};
+  mb.compose = 0;
+  mb.nmat = nmat;
+  std::memcpy(mb.u.M, N, sizeof(double) * 9 * nmat);
+  return binmd_run(g, mb, nevents, events, stride_floats, col_w, col_q, (cudaStream_t)stream);
+}
+
+mdn_status mdnorm_debug_trajectories(mdn_grid* g, int32_t nmat, const double* M, const double* charge,
+                                     double k_min, double k_max, int64_t ntraj, const int64_t* traj_ids,
+                                     int32_t* n_cross, int32_t* n_seg, int64_t* seg_bins, double* seg_vals,
+                                     int64_t max_segs) {
+  mdn_status st;
+  if ((st = check_ready(g)) != MDN_OK) return st;
+  if (nmat < 1 || nmat > MDN_MAX_MATS || !M || !charge) return fail(MDN_EINVAL, "nmat %d outside [1, %d]", nmat, MDN_MAX_MATS);
+  if ((st = check_krange(k_min, k_max)) != MDN_OK) return st;
+  if (ntraj < 0 || max_segs < 0 || (ntraj > 0 && (!traj_ids || !n_cross || !n_seg)) ||
+      (max_segs > 0 && ntraj > 0 && (!seg_bins || !seg_vals)))
+    return fail(MDN_EINVAL, "bad debug arguments");
+  for (int64_t t = 0; t < ntraj; ++t)
+    if (traj_ids[t] < 0 || traj_ids[t] >= (int64_t)nmat * g->npix) return fail(MDN_EINVAL, "traj id %lld out of range", (long long)traj_ids[t]);
+  if (ntraj == 0) return ok();
+  DeviceGuard dg(g->device);
+  MatBlock mb{};
+  mb.compose = 0;
+  mb.nmat = nmat;
+  std::memcpy(mb.u.M, M, sizeof(double) * 9 * nmat);
+  std::memcpy(mb.charge, charge, sizeof(double) * nmat);
+  const int64_t ms = std::max<int64_t>(max_segs, 1);
+  int64_t* d_ids = nullptr;
+  int32_t* d_nc = nullptr;
+  int32_t* d_ns = nullptr;
+  int64_t* d_bins = nullptr;
+  double* d_vals = nullptr;
+  cudaError_t e = cudaMalloc(&d_ids, sizeof(int64_t) * ntraj);
+  if (e == cudaSuccess) e = cudaMalloc(&d_nc, sizeof(int32_t) * ntraj);
+  if (e == cudaSuccess) e = cudaMalloc(&d_ns, sizeof(int32_t) * ntraj);
+  if (e == cudaSuccess) e = cudaMalloc(&d_bins, sizeof(int64_t) * ntraj * ms);
+  if (e == cudaSuccess) e = cudaMalloc(&d_vals, sizeof(double) * ntraj * ms);
+  if (e == cudaSuccess) e = cudaMemcpy(d_ids, traj_ids, sizeof(int64_t) * ntraj, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess)
+    e = mdn::launch_debug_traj(mdn_params(g, k_min, k_max, 0, 1, 0), mb, ntraj, d_ids, g->npix, d_nc, d_ns, d_bins,
+                               d_vals, max_segs, nullptr);
+  if (e == cudaSuccess) e = cudaDeviceSynchronize();
+  if (e == cudaSuccess) e = cudaMemcpy(n_cross, d_nc, sizeof(int32_t) * ntraj, cudaMemcpyDeviceToHost);
+  if (e == cudaSuccess) e = cudaMemcpy(n_seg, d_ns, sizeof(int32_t) * ntraj, cudaMemcpyDeviceToHost);
+  if (e == cudaSuccess && max_segs > 0) e = cudaMemcpy(seg_bins, d_bins, sizeof(int64_t) * ntraj * max_segs, cudaMemcpyDeviceToHost);
+  if (e == cudaSuccess && max_segs > 0) e = cudaMemcpy(seg_vals, d_vals, sizeof(double) * ntraj * max_segs, cudaMemcpyDeviceToHost);
+  cudaFree(d_ids);
+  cudaFree(d_nc);
+  cudaFree(d_ns);
+  cudaFree(d_bins);
+  cudaFree(d_vals);
+  if (e != cudaSuccess) return cuda_fail(e, "debug trajectories");
+  return ok();
+}
+
+mdn_status binmd_debug_bins(mdn_grid* g, int32_t nmat, const double* N, int64_t nevents, const float* events,
+                            int64_t stride_floats, int32_t col_w, int32_t col_q, int64_t* bins) {
+  if (!g) return fail(MDN_EINVAL, "grid is NULL");
+  if (nmat < 1 || nmat > MDN_MAX_MATS || !N || !bins) return fail(MDN_EINVAL, "bad debug arguments");
+  mdn_status st;
+  if ((st = check_events(nevents, events, stride_floats, col_w, col_q)) != MDN_OK) return st;
+  if (nevents == 0) return ok();
+  DeviceGuard dg(g->device);
+  MatBlock mb{};
+  mb.compose = 0;
+  mb.nmat = nmat;
+  std::memcpy(mb.u.M, N, sizeof(double) * 9 * nmat);
+  float* d_ev = nullptr;
+  int64_t* d_bins = nullptr;
+  const bool dev = is_device_ptr(events);
+  cudaError_t e = cudaSuccess;
+  if (!dev) {
+    e = cudaMalloc(&d_ev, sizeof(float) * nevents * stride_floats);
+    if (e == cudaSuccess) e = cudaMemcpy(d_ev, events, sizeof(float) * nevents * stride_floats, cudaMemcpyHostToDevice);
+  }
+  if (e == cudaSuccess) e = cudaMalloc(&d_bins, sizeof(int64_t) * nevents * nmat);
+  if (e == cudaSuccess)
+    e = mdn::launch_debug_bins(bin_params(g, dev ? events : d_ev, nevents, stride_floats, col_w, col_q), mb, d_bins,
+                               nullptr);
+  if (e == cudaSuccess) e = cudaDeviceSynchronize();
+  if (e == cudaSuccess) e = cudaMemcpy(bins, d_bins, sizeof(int64_t) * nevents * nmat, cudaMemcpyDeviceToHost);
+  cudaFree(d_ev);
+  cudaFree(d_bins);
+  if (e != cudaSuccess) return cuda_fail(e, "debug bins");
+  return ok();
+}
+
+mdn_status mdnorm_debug_compose(mdn_grid* g, const double UB[9], int32_t nruns, const double* R, int32_t nops,
+                                const double* ops, double* M, double* N) {
+  if (!g) return fail(MDN_EINVAL, "grid is NULL");
+  mdn_status st;
+  if ((st = check_matrix(UB, "UB")) != MDN_OK) return st;
+  if ((st = check_ops(nops, ops)) != MDN_OK) return st;
+  if (nruns < 1 || nruns > mdn::kRunsPerLaunch || !R || !M || !N) return fail(MDN_EINVAL, "bad debug arguments");
+  DeviceGuard dg(g->device);
+  MatBlock a{}, b{};
+  a.compose = b.compose = 1;
+  a.nops = b.nops = nops;
+  a.nruns = nruns;
+  a.nmat = nruns * nops;
+  b.nmat = nops;
+  std::memcpy(a.UB, UB, sizeof a.UB);
+  std::memcpy(b.UB, UB, sizeof b.UB);
+  std::memcpy(a.W, g->W, sizeof a.W);
+  std::memcpy(b.W, g->W, sizeof b.W);
+  std::memcpy(a.u.c.ops, ops, sizeof(double) * 9 * nops);
+  std::memcpy(b.u.c.ops, ops, sizeof(double) * 9 * nops);
+  std::memcpy(a.u.c.R, R, sizeof(double) * 9 * nruns);
+  double *dM = nullptr, *dN = nullptr;
+  int32_t* dok = nullptr;
+  int32_t hok = 1;
+  cudaError_t e = cudaMalloc(&dM, sizeof(double) * 9 * a.nmat);
+  if (e == cudaSuccess) e = cudaMalloc(&dN, sizeof(double) * 9 * nops);
+  if (e == cudaSuccess) e = cudaMalloc(&dok, sizeof(int32_t));
+  if (e == cudaSuccess) e = cudaMemcpy(dok, &hok, sizeof hok, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = mdn::launch_debug_compose(a, b, dM, dN, dok, nullptr);
+  if (e == cudaSuccess) e = cudaDeviceSynchronize();
+  if (e == cudaSuccess) e = cudaMemcpy(M, dM, sizeof(double) * 9 * a.nmat, cudaMemcpyDeviceToHost);
+  if (e == cudaSuccess) e = cudaMemcpy(N, dN, sizeof(double) * 9 * nops, cudaMemcpyDeviceToHost);
+  if (e == cudaSuccess) e = cudaMemcpy(&hok, dok, sizeof hok, cudaMemcpyDeviceToHost);
+  cudaFree(dM);
+  cudaFree(dN);
+  cudaFree(dok);
+  if (e != cudaSuccess) return cuda_fail(e, "debug compose");
+  if (!hok) return fail(MDN_EINVAL, "a composed matrix is singular");
+  return ok();
+}
+
+}  // extern "C"

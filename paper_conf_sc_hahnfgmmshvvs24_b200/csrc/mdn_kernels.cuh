@@ -1,0 +1,72 @@
+// mdn_kernels.cuh -- launch parameter blocks and launcher declarations (internal, not the ABI).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "mdn_device.cuh"
+
+namespace mdn {
+
+constexpr int kMaxOps = 48;           // MDN_MAX_OPS
+constexpr int kMaxMats = 64;          // MDN_MAX_MATS
+constexpr int kRunsPerLaunch = 16;    // runs composed per MDNorm launch (batched API)
+constexpr int kFluxSmemMax = 4096;    // flux knots staged in shared memory (64 KB fp64 pairs)
+
+// Matrices for one launch, passed by value as a __grid_constant__ kernel parameter (sm_70+
+// kernels accept up to 32 KB of parameters; CUDA >= 12.1).  Either compose (UB, W, ops, R) on
+// the device (API mode, M0/B0) or take final matrices (parity mode).
+struct MatBlock {
+  int32_t compose;   // 1: compose from UB/W/ops/R; 0: use M
+  int32_t nops;      // compose mode
+  int32_t nruns;     // compose mode (MDNorm); 0 for BinMD
+  int32_t nmat;      // = nruns * nops (MDNorm), nops (BinMD), or the parity count
+  double UB[9];
+  double W[9];
+  double charge[kMaxMats > kRunsPerLaunch ? kMaxMats : kRunsPerLaunch];  // per run / per matrix
+  union {
+    struct {
+      double ops[kMaxOps * 9];
+      double R[kRunsPerLaunch * 9];
+    } c;
+    double M[kMaxMats * 9];
+  } u;
+};
+
+struct MdnParams {
+  GridC g;
+  const double4* pix;      // (q0, q1, q2, Omega) per pixel, q = z - d  (M1)
+  int64_t pix_begin, pix_stride, nshard;
+  const double* flux_k;
+  const double* flux_F;
+  int32_t nflux;
+  int32_t acc_f32;
+  double kmin, kmax;
+  double* norm;            // fp64 histogram (nbins)
+  unsigned long long* stats;  // nullptr, or [traj, hits, crossings, segments] (+= per launch)
+};
+
+struct BinParams {
+  GridC g;
+  const float* events;
+  int64_t nevents, stride;
+  int32_t col_w, col_q;
+  int32_t acc_f32;
+  double* binmd;           // fp64 histogram (nbins)
+  unsigned long long* stats;  // nullptr, or [pairs, inside] (+= per launch)
+};
+
+// launchers (return the launch's cudaError_t)
+cudaError_t launch_pixels_prepare(const double* dir, const double* solid, double4* pix, int64_t npix,
+                                  cudaStream_t s);
+cudaError_t launch_mdnorm(const MdnParams& p, const MatBlock& mb, int num_sms, cudaStream_t s);
+cudaError_t launch_binmd(const BinParams& p, const MatBlock& mb, int num_sms, cudaStream_t s);
+cudaError_t launch_cross_section(const double* norm, const double* binmd, double* xs, int64_t nbins,
+                                 int num_sms, cudaStream_t s);
+cudaError_t launch_debug_traj(const MdnParams& p, const MatBlock& mb, int64_t ntraj,
+                              const int64_t* ids, int64_t npix, int32_t* n_cross, int32_t* n_seg,
+                              int64_t* seg_bins, double* seg_vals, int64_t max_segs, cudaStream_t s);
+cudaError_t launch_debug_bins(const BinParams& p, const MatBlock& mb, int64_t* bins, cudaStream_t s);
+cudaError_t launch_debug_compose(const MatBlock& mdn, const MatBlock& bin, double* M, double* N,
+                                 int32_t* ok, cudaStream_t s);
+
+}  // namespace mdn

@@ -1,0 +1,76 @@
+"""N > 1 host logic on CPU: world_size-2 gloo processes follow the shard plan,
+compute their partial histograms (with the oracle standing in for the GPU kernels -- test
+only), pack [norm | binmd] and make ONE reduce; rank 0 must obtain the single-process result."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+from paper_conf_sc_hahnfgmmshvvs24_b200.dist import plan_shards, reduce_packed
+
+
+def test_plan_covers_everything_once():
+    for world in (1, 2, 3, 8):
+        # multi-run: run blocks
+        runs = sorted(r for k in range(world) for r in plan_shards(world, k, 120, 1000, 10).runs)
+        assert runs == list(range(120))
+        # single run: interleaved pixels and contiguous event blocks
+        pix = sorted(p for k in range(world) for p in range(plan_shards(world, k, 1, 1000, 10).pix_begin,
+                                                                   1000, plan_shards(world, k, 1, 1000, 10).pix_stride))
+        assert pix == list(range(1000))
+        ev = [plan_shards(world, k, 1, 1000, 1001).event_ranges[0] for k in range(world)]
+        assert ev[0][0] == 0 and ev[-1][1] == 1001
+        assert all(ev[i][1] == ev[i + 1][0] for i in range(world - 1))
+    with pytest.raises(ValueError):
+        plan_shards(2, 2, 1, 10, 10)
+
+
+def _free_port():
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def _worker(rank, world, port, out):
+    import oracle
+    import synth
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    wl = synth.make_workload("tiny", events_per_run=5000)
+    wl.ops = synth.hex_6mmm_ops()[:4]
+    g = oracle.workload_grid(wl)
+    ev = synth.events_for_run(wl, 0)
+    p = plan_shards(world, rank, wl.nruns, wl.npix, len(ev))
+    M = oracle.mdnorm_matrices(wl.R, wl.UB, wl.ops, wl.W)
+    norm = oracle.mdnorm(g, wl.pix_dir, wl.solid, wl.flux_k, wl.flux_F, M, 1.0, wl.k_min, wl.k_max,
+                         pix_begin=p.pix_begin, pix_stride=p.pix_stride)
+    b, e = p.event_ranges[0]
+    bm = oracle.binmd(g, oracle.binmd_matrices(wl.UB, wl.ops, wl.W), ev[b:e])
+    packed = torch.from_numpy(np.concatenate([norm, bm]))
+    reduce_packed(packed, dst=0)
+    if rank == 0:
+        full_n, full_b, _ = oracle.run_workload(wl, events={0: ev})
+        n = g.nbins
+        out.put((np.abs(packed[:n].numpy() - full_n).max() / full_n.max(),
+                 float(np.abs(packed[n:].numpy() - full_b).max())))
+    dist.destroy_process_group()
+
+
+def test_gloo_world2_reduce_matches_single_process():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    rel_n, abs_b = q.get(timeout=300)
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert rel_n < 1e-14
+    assert abs_b == 0.0  # unit weights: integer counts add exactly
