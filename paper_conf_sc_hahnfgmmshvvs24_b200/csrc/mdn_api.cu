@@ -25,8 +25,13 @@ struct mdn_grid {
   double* d_hist = nullptr;  // [norm | binmd], 2 * nbins doubles
   double4* d_pix = nullptr;
   int64_t npix = 0;
-  double* d_flux = nullptr;  // [k | F], 2 * nflux doubles
-  int32_t nflux = 0;
+  double2* d_flux = nullptr;  // (kappa_i, Phi_i), nflux entries
+  int* d_ftab = nullptr;      // flux search start table (nftab cells)
+  int32_t nflux = 0, nftab = 0;
+  double ftab_k0 = 0.0, ftab_inv_cell = 0.0;
+  mdn::Hitter* d_hit = nullptr;       // cull -> walk hand-off buffer
+  uint32_t hit_cap = 0;
+  mdn::DevCounters* d_ctr = nullptr;
   double* d_xs = nullptr;    // scratch for host xs
   unsigned long long* d_stats = nullptr;  // 6 work counters (mdnorm_stats)
   bool stats_on = false;
@@ -163,15 +168,52 @@ mdn::MdnParams mdn_params(mdn_grid* g, double k_min, double k_max, int64_t pix_b
   p.pix_begin = pix_begin;
   p.pix_stride = pix_stride;
   p.nshard = nshard;
-  p.flux_k = g->d_flux;
-  p.flux_F = g->d_flux + g->nflux;
-  p.nflux = g->nflux;
+  p.flux.kf = g->d_flux;
+  p.flux.tab = g->d_ftab;
+  p.flux.k0 = g->ftab_k0;
+  p.flux.inv_cell = g->ftab_inv_cell;
+  p.flux.n = g->nflux;
+  p.flux.ntab = g->nftab;
   p.acc_f32 = g->acc == MDN_ACC_F32;
   p.kmin = k_min;
   p.kmax = k_max;
   p.norm = g->d_hist;
   p.stats = g->stats_on ? g->d_stats : nullptr;
+  p.hit = g->d_hit;
+  p.ctr = g->d_ctr;
   return p;
+}
+
+constexpr uint32_t kMaxSlab = 1u << 24;  // trajectories per cull/walk pair (1 GiB hitter buffer)
+
+// MDNorm over all nmat x nshard trajectories of one launch block: slabs of at most kMaxSlab
+// trajectories, each a cull kernel (compacting hitters into g->d_hit) and a walk kernel.  The
+// hitter buffer holds one slab's worst case (every trajectory hits), so no count ever has to
+// come back to the host (the MiniVATES host round trip of P:139 is avoided).
+mdn_status run_mdnorm(mdn_grid* g, mdn::MdnParams p, const MatBlock& mb, cudaStream_t s) {
+  const uint64_t ntraj = (uint64_t)mb.nmat * (uint64_t)p.nshard;
+  if (ntraj == 0) return MDN_OK;
+  if (ntraj >= (1ull << 32)) return fail(MDN_EINVAL, "too many trajectories in one launch (%llu)", (unsigned long long)ntraj);
+  const uint32_t want = (uint32_t)std::min<uint64_t>(ntraj, kMaxSlab);
+  if (g->hit_cap < want) {
+    if (g->d_hit) {
+      cudaStreamSynchronize(s);
+      cudaFree(g->d_hit);
+    }
+    g->d_hit = nullptr;
+    g->hit_cap = 0;
+    MDN_CUDA(cudaMalloc(&g->d_hit, sizeof(mdn::Hitter) * (size_t)want), "hitter buffer");
+    g->hit_cap = want;
+  }
+  if (!g->d_ctr) MDN_CUDA(cudaMalloc(&g->d_ctr, sizeof(mdn::DevCounters)), "counters");
+  p.hit = g->d_hit;
+  p.ctr = g->d_ctr;
+  for (uint64_t t0 = 0; t0 < ntraj; t0 += g->hit_cap) {
+    p.t0 = (uint32_t)t0;
+    p.tlen = (uint32_t)std::min<uint64_t>(g->hit_cap, ntraj - t0);
+    MDN_CUDA(mdn::launch_mdnorm(p, mb, g->num_sms, s), "mdnorm kernels");
+  }
+  return MDN_OK;
 }
 
 mdn_status check_events(int64_t nevents, const float* events, int64_t stride, int32_t col_w, int32_t col_q) {
@@ -311,6 +353,9 @@ mdn_status mdnorm_destroy(mdn_grid* g) {
   cudaFree(g->d_hist);
   cudaFree(g->d_pix);
   cudaFree(g->d_flux);
+  cudaFree(g->d_ftab);
+  cudaFree(g->d_hit);
+  cudaFree(g->d_ctr);
   cudaFree(g->d_xs);
   cudaFree(g->d_stats);
   for (int i = 0; i < 2; ++i) {
@@ -367,18 +412,31 @@ mdn_status mdnorm_set_flux(mdn_grid* g, int64_t n, const double* k, const double
     if (!(hk[i] > hk[i - 1])) return fail(MDN_EINVAL, "flux k not strictly increasing at %lld", (long long)i);
     if (hF[i] < hF[i - 1]) return fail(MDN_EINVAL, "cumulative flux F decreases at %lld", (long long)i);
   }
-  double* d = nullptr;
-  cudaError_t e = cudaMalloc(&d, sizeof(double) * 2 * n);
-  if (e == cudaSuccess) e = cudaMemcpy(d, hk.data(), sizeof(double) * n, cudaMemcpyHostToDevice);
-  if (e == cudaSuccess) e = cudaMemcpy(d + n, hF.data(), sizeof(double) * n, cudaMemcpyHostToDevice);
+  // (kappa_i, Phi_i) interleaved, plus the search start table of flux_at (M5): 2n uniform cells
+  std::vector<double2> kf((size_t)n);
+  for (int64_t i = 0; i < n; ++i) kf[i] = make_double2(hk[i], hF[i]);
+  const int ntab = (int)std::min<int64_t>(2 * n, 1 << 22);
+  const double cell = (hk[n - 1] - hk[0]) / (double)ntab;
+  double2* d = nullptr;
+  int* tab = nullptr;
+  cudaError_t e = cudaMalloc(&d, sizeof(double2) * n);
+  if (e == cudaSuccess) e = cudaMalloc(&tab, sizeof(int) * ntab);
+  if (e == cudaSuccess) e = cudaMemcpy(d, kf.data(), sizeof(double2) * n, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = mdn::launch_flux_table(d, (int)n, tab, ntab, hk[0], cell, nullptr);
+  if (e == cudaSuccess) e = cudaDeviceSynchronize();
   if (e != cudaSuccess) {
     cudaFree(d);
+    cudaFree(tab);
     return cuda_fail(e, "set_flux");
   }
-  cudaDeviceSynchronize();
   cudaFree(g->d_flux);
+  cudaFree(g->d_ftab);
   g->d_flux = d;
+  g->d_ftab = tab;
   g->nflux = (int32_t)n;
+  g->nftab = ntab;
+  g->ftab_k0 = hk[0];
+  g->ftab_inv_cell = 1.0 / cell;
   return ok();
 }
 
@@ -414,7 +472,7 @@ mdn_status mdnorm_accumulate_runs(mdn_grid* g, const double UB[9], int32_t nruns
     std::memcpy(mb.u.c.ops, ops, sizeof(double) * 9 * nops);
     std::memcpy(mb.u.c.R, R + 9 * r0, sizeof(double) * 9 * nr);
     std::memcpy(mb.charge, charge + r0, sizeof(double) * nr);
-    MDN_CUDA(mdn::launch_mdnorm(p, mb, g->num_sms, s), "mdnorm kernel");
+    if ((st = run_mdnorm(g, p, mb, s)) != MDN_OK) return st;
   }
   return ok();
 }
@@ -515,8 +573,9 @@ mdn_status mdnorm_accumulate_matrices(mdn_grid* g, int32_t nmat, const double* M
   mb.nmat = nmat;
   std::memcpy(mb.u.M, M, sizeof(double) * 9 * nmat);
   std::memcpy(mb.charge, charge, sizeof(double) * nmat);
-  MDN_CUDA(mdn::launch_mdnorm(mdn_params(g, k_min, k_max, pix_begin, pix_stride, nshard), mb, g->num_sms,
-                              (cudaStream_t)stream), "mdnorm kernel");
+  if ((st = run_mdnorm(g, mdn_params(g, k_min, k_max, pix_begin, pix_stride, nshard), mb, (cudaStream_t)stream)) !=
+      MDN_OK)
+    return st;
   return ok();
 }
 

@@ -1,10 +1,10 @@
 // mdn_device.cuh -- device-side building blocks of the MDNorm / BinMD hot path (sm_100a).
 //
-// Every function here is IEEE fp64 with explicit round-to-nearest intrinsics (__dmul_rn,
-// __dadd_rn, __dsub_rn, __ddiv_rn), so no multiply-add is ever contracted into an FMA and the
-// crossing values, midpoints, bin indices and flux values are bit-identical to the paper's
+// Every value that decides a crossing, a clip, a midpoint, a bin index or a flux value is IEEE
+// fp64 with explicit round-to-nearest intrinsics (__dmul_rn, __dadd_rn, __ddiv_rn), so no
+// multiply-add is ever contracted into an FMA and the results are bit-identical to the paper's
 // definition as DESIGN.md §3 fixes it.  The translation unit is
-// additionally compiled with --fmad=false as a guard.
+// also compiled with --fmad=false as a guard.
 //
 // Citations: PAPER.md P:n.  M0-M7, B0-B3, X2 = the rows of SURVEY.md §8(a).
 #pragma once
@@ -15,8 +15,8 @@
 namespace mdn {
 
 // ------------------------------------------------------------------------------ grid constants
-// w_a = (hi_a - lo_a) / n_a, s_a = 1 / w_a, computed once on the host in IEEE double (identical
-// to the device result; x86-64 SSE2).  Edge e_{a,j} = lo_a + j * w_a (product, then sum).
+// w_a = (hi_a - lo_a) / n_a, s_a = 1 / w_a, computed once on the host in IEEE double (x86-64
+// SSE2: the same bits the device would produce).  Edge e_{a,j} = lo_a + j * w_a.
 struct GridC {
   double lo[3], hi[3], w[3], s[3];
   int32_t n[3];
@@ -92,27 +92,34 @@ __device__ __forceinline__ bool compose_binmd(const double* UB, const double* S,
 }
 
 // ------------------------------------------------------------------------------ M5 flux
-// F(x): clamp outside, else i = max{i : k_i <= x} (unique, so any search order gives the same i)
-// and Phi_i + (Phi_{i+1} - Phi_i) * ((x - k_i) / (k_{i+1} - k_i)).
+// F(x): clamp outside, else i = max{i : kappa_i <= x} and
+//   Phi_i + (Phi_{i+1} - Phi_i) * ((x - kappa_i) / (kappa_{i+1} - kappa_i)).
+// i is unique, so it may be found by any search: here a uniform-cell index table gives a start
+// index that is then corrected by exact comparisons (O(1) expected instead of a 12-step binary
+// search).  tab[c] = max{i : kappa_i <= kappa_0 + c * cell} (setup kernel; any monotone guess
+// would do because the loops below fix it).
 struct FluxView {
-  const double* k;
-  const double* F;
-  int n;
+  const double2* kf;  // (kappa_i, Phi_i)
+  const int* tab;     // ntab cell start indices
+  double k0, inv_cell;
+  int n, ntab;
 };
 
 __device__ __forceinline__ double flux_at(const FluxView& f, double x) {
-  if (x <= f.k[0]) return f.F[0];
-  if (x >= f.k[f.n - 1]) return f.F[f.n - 1];
-  int lo = 0, hi = f.n - 1;  // invariant k[lo] <= x < k[hi]
-  while (hi - lo > 1) {
-    int mid = (lo + hi) >> 1;
-    if (f.k[mid] <= x)
-      lo = mid;
-    else
-      hi = mid;
+  const double2 first = f.kf[0], last = f.kf[f.n - 1];
+  if (x <= first.x) return first.y;
+  if (x >= last.x) return last.y;
+  double u = (x - first.x) * f.inv_cell;  // any rounding: only a starting guess
+  int c = u < (double)f.ntab ? (int)u : f.ntab - 1;
+  int i = f.tab[c < 0 ? 0 : c];
+  while (i > 0 && f.kf[i].x > x) --i;
+  double2 lo = f.kf[i], hi = f.kf[i + 1];
+  while (hi.x <= x) {  // terminates: x < kappa_{n-1}
+    ++i;
+    lo = hi;
+    hi = f.kf[i + 1];
   }
-  double k0 = f.k[lo], k1 = f.k[lo + 1], F0 = f.F[lo], F1 = f.F[lo + 1];
-  return dadd(F0, dmul(dsub(F1, F0), ddiv(dsub(x, k0), dsub(k1, k0))));
+  return dadd(lo.y, dmul(dsub(hi.y, lo.y), ddiv(dsub(x, lo.x), dsub(hi.x, lo.x))));
 }
 
 // ------------------------------------------------------------------------------ M1-M2
@@ -143,12 +150,12 @@ __device__ __forceinline__ bool traj_clip(const GridC& g, const double v[3], dou
 }
 
 // ------------------------------------------------------------------------------ M3
-// Plane crossings of axis a: J = {j in [1, n-1] : kin < e_j * r < kout} with r = 1/v.
+// Plane crossings of axis a: J = {j in [1, n-1] : lo_k < e_j * r < hi_k} with r = 1/v.
 // f(j) = e_j * r is monotone in j (rounding is monotone), so J is one contiguous index range:
 // the region-of-interest replacement of the paper's linear plane loops.
 // The range is estimated from the continuous grid coordinate and fixed up by exact tests of
-// f(j) itself, so J is exactly the oracle's set.  Output: first index in increasing-k order,
-// count, and step (+1 if v > 0, -1 if v < 0).
+// f(j) itself, so J is exactly the oracle's set.  The stream yields J in increasing k:
+// first index j, count cnt, step +1 (v > 0) or -1 (v < 0).
 struct AxisStream {
   int j, cnt, step;
 };
@@ -183,9 +190,8 @@ __device__ __forceinline__ AxisStream axis_stream(const GridC& g, int a, double 
     j = clamp_floor(u_out, 0, n - 1);
     while (j < n - 1 && plane_k(g, a, j + 1, r) < kout) ++j;
     while (j >= 1 && !(plane_k(g, a, j, r) < kout)) --j;
-    int jhi = j;
     s.j = jlo;
-    s.cnt = jhi >= jlo ? jhi - jlo + 1 : 0;
+    s.cnt = j >= jlo ? j - jlo + 1 : 0;
     s.step = 1;
   } else {
     // f decreasing: increasing k visits descending j.  jA = last j with f(j) > kin.
@@ -197,62 +203,83 @@ __device__ __forceinline__ AxisStream axis_stream(const GridC& g, int a, double 
     j = clamp_floor(u_out + 1.0, 1, n);
     while (j > 1 && plane_k(g, a, j - 1, r) < kout) --j;
     while (j <= n - 1 && !(plane_k(g, a, j, r) < kout)) ++j;
-    int jB = j;
     s.j = jA;
-    s.cnt = jA >= jB ? jA - jB + 1 : 0;
+    s.cnt = jA >= j ? jA - j + 1 : 0;
     s.step = -1;
   }
   return s;
 }
 
+// One axis of the merge: reciprocal, position in its stream, next crossing value.
+struct AxisCursor {
+  double r, nk;
+  int j, cnt, step;
+};
+
+__device__ __forceinline__ void cursor_init(AxisCursor& c, const GridC& g, int a, double v, double lo_k,
+                                            double hi_k) {
+  c.r = v != 0.0 ? ddiv(1.0, v) : 0.0;
+  const AxisStream s = axis_stream(g, a, v, c.r, lo_k, hi_k);
+  c.j = s.j;
+  c.cnt = s.cnt;
+  c.step = s.step;
+  c.nk = s.cnt > 0 ? plane_k(g, a, s.j, c.r) : CUDART_INF;
+}
+
+__device__ __forceinline__ void cursor_advance(AxisCursor& c, const GridC& g, int a) {
+  c.cnt -= 1;
+  c.j += c.step;
+  c.nk = c.cnt > 0 ? plane_k(g, a, c.j, c.r) : CUDART_INF;
+}
+
 // ------------------------------------------------------------------------------ M4-M7
-// Walk one clipped trajectory: a 3-way streaming merge of the per-axis monotone crossing
-// sequences (replaces the paper's sort, and the GPU comb sort, with no buffer),
-// flux at each list entry (M5), midpoint bin of every positive-length segment (M6) and
-// emit(b, (F(k2) - F(k1)) * omega_c) (M7).  Returns n_seg; *ncross = |L| = 2 + crossings.
+// Walk the part [lo_k, hi_k] of a clipped trajectory, where lo_k and hi_k are members of the
+// trajectory's list L (its clip endpoints or plane crossings): a 3-way streaming merge of the
+// per-axis monotone crossing sequences strictly inside (lo_k, hi_k) (replaces the paper's sort,
+// P:115, and the GPU comb sort, with no buffer), flux at each list entry (M5), midpoint
+// bin of every positive-length segment (M6) and emit(b, (F(k2) - F(k1)) * omega_c) (M7).
+// Splitting L at any of its members leaves the set of segments unchanged, which is what lets
+// the production kernel cut long trajectories into balanced pieces.  Returns n_seg; *ncross
+// receives the number of crossings strictly inside (lo_k, hi_k).
 template <class Emit>
-__device__ __forceinline__ int traj_walk(const GridC& g, const FluxView& fx, const double v[3],
-                                         double kin, double kout, double omega_c, Emit& emit,
-                                         int* ncross) {
-  double r[3], nk[3];
-  AxisStream st[3];
-  int total = 0;
-#pragma unroll
-  for (int a = 0; a < 3; ++a) {
-    r[a] = v[a] != 0.0 ? ddiv(1.0, v[a]) : 0.0;
-    st[a] = axis_stream(g, a, v[a], r[a], kin, kout);
-    total += st[a].cnt;
-    nk[a] = st[a].cnt > 0 ? plane_k(g, a, st[a].j, r[a]) : CUDART_INF;
-  }
-  *ncross = total + 2;
-  double k1 = kin, F1 = flux_at(fx, kin);
+__device__ __forceinline__ int traj_walk(const GridC& g, const FluxView& fx, double v0, double v1,
+                                         double v2, double lo_k, double hi_k, double omega_c,
+                                         Emit& emit, int* ncross) {
+  AxisCursor c0, c1, c2;
+  cursor_init(c0, g, 0, v0, lo_k, hi_k);
+  cursor_init(c1, g, 1, v1, lo_k, hi_k);
+  cursor_init(c2, g, 2, v2, lo_k, hi_k);
+  const int total = c0.cnt + c1.cnt + c2.cnt;
+  *ncross = total;
+  double k1 = lo_k, F1 = flux_at(fx, lo_k);
   int nseg = 0;
   for (int left = total;; --left) {
     double k2;
     if (left > 0) {
-      int a = 0;
-      k2 = nk[0];
-      if (nk[1] < k2) { a = 1; k2 = nk[1]; }
-      if (nk[2] < k2) { a = 2; k2 = nk[2]; }
-      st[a].cnt -= 1;
-      st[a].j += st[a].step;
-      nk[a] = st[a].cnt > 0 ? plane_k(g, a, st[a].j, r[a]) : CUDART_INF;
+      if (c0.nk <= c1.nk && c0.nk <= c2.nk) {
+        k2 = c0.nk;
+        cursor_advance(c0, g, 0);
+      } else if (c1.nk <= c2.nk) {
+        k2 = c1.nk;
+        cursor_advance(c1, g, 1);
+      } else {
+        k2 = c2.nk;
+        cursor_advance(c2, g, 2);
+      }
     } else {
-      k2 = kout;
+      k2 = hi_k;
     }
     if (k2 > k1) {
-      double F2 = flux_at(fx, k2);
-      double km = dmul(0.5, dadd(k1, k2));
-      bool inside = true;
-      int idx[3];
-#pragma unroll
-      for (int a = 0; a < 3; ++a) {
-        double t = dmul(dsub(dmul(km, v[a]), g.lo[a]), g.s[a]);
-        inside = inside && (0.0 <= t && t < (double)g.n[a]);
-        idx[a] = __double2int_rz(t);
-      }
-      if (inside) {
-        int64_t b = (int64_t)idx[0] + (int64_t)g.n[0] * ((int64_t)idx[1] + (int64_t)g.n[1] * idx[2]);
+      const double F2 = flux_at(fx, k2);
+      const double km = dmul(0.5, dadd(k1, k2));
+      const double t0 = dmul(dsub(dmul(km, v0), g.lo[0]), g.s[0]);
+      const double t1 = dmul(dsub(dmul(km, v1), g.lo[1]), g.s[1]);
+      const double t2 = dmul(dsub(dmul(km, v2), g.lo[2]), g.s[2]);
+      if (0.0 <= t0 && t0 < (double)g.n[0] && 0.0 <= t1 && t1 < (double)g.n[1] && 0.0 <= t2 &&
+          t2 < (double)g.n[2]) {
+        const int64_t b = (int64_t)__double2int_rz(t0) +
+                          (int64_t)g.n[0] * ((int64_t)__double2int_rz(t1) +
+                                             (int64_t)g.n[1] * __double2int_rz(t2));
         emit(b, dmul(dsub(F2, F1), omega_c));
         ++nseg;
       }

@@ -1,8 +1,17 @@
 // mdn_kernels.cu -- sm_100a kernels of the MDNorm / BinMD cross-section hot path.
 //
-// Rows of SURVEY.md §8(a):  M0 compose (prologue of mdnorm_kernel), M1-M7 mdnorm_kernel,
-// B0 compose (prologue of binmd_kernel), B1-B3 binmd_kernel, X2 xs_kernel.  The parity entry
-// points (debug_*) run the very same device functions (mdn_device.cuh).
+// Rows of SURVEY.md §8(a):
+//   M0 compose        prologue of mdnorm_cull_kernel / debug kernels (matrices in smem)
+//   M1-M3 (cull)      mdnorm_cull_kernel: one thread per trajectory (pixel x op x run): v, clip,
+//                     per-axis crossing ranges; hitters are compacted (warp ballot + one atomic
+//                     per warp) into a hitter list with their piece plan
+//   M3-M7 (walk)      mdnorm_walk_kernel: persistent warps claim batches of 32 hitters, cut them
+//                     into pieces of ~kPieceSegs segments at crossings of the busiest axis, and
+//                     every lane walks one piece (streaming 3-way merge, flux from smem, midpoint
+//                     bin, fp64 red.add into the L2-resident histogram)
+//   B0-B3             binmd_kernel (compose prologue, streaming event loads, ops in smem)
+//   X2                xs_kernel
+// The parity entry points (debug_*) run the very same device functions (mdn_device.cuh).
 #include <algorithm>
 
 #include "mdn_kernels.cuh"
@@ -12,6 +21,8 @@ namespace mdn {
 namespace {
 
 constexpr int kThreads = 256;
+constexpr int kWalkThreads = 512;
+constexpr unsigned kFull = 0xffffffffu;
 
 __device__ __forceinline__ void stage_mdnorm_mats(const MatBlock& mb, double* sM, double* sC) {
   for (int m = threadIdx.x; m < mb.nmat; m += blockDim.x) {
@@ -41,7 +52,7 @@ __device__ __forceinline__ void stage_binmd_mats(const MatBlock& mb, double* sN)
 // One warp-aggregated atomic per counter per warp (tracing only; compiled out when kStats off).
 __device__ __forceinline__ void flush_counter(unsigned long long* dst, unsigned long long v) {
 #pragma unroll
-  for (int o = 16; o > 0; o >>= 1) v += __shfl_down_sync(0xffffffffu, v, o);
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_down_sync(kFull, v, o);
   if ((threadIdx.x & 31) == 0 && v) atomicAdd(dst, v);
 }
 
@@ -50,43 +61,72 @@ struct AtomicEmit {
   __device__ __forceinline__ void operator()(int64_t b, double val) const { atomicAdd(h + b, val); }
 };
 
-// ---------------------------------------------------------------- M1-M7: one thread per pixel,
-// looping over every (run, op) matrix of the launch (pixel read once, P:102 collapse(2) space).
-template <bool kSmemFlux, bool kStats>
+// ---------------------------------------------------------------- M1-M3: cull + compaction
+template <bool kStats>
 __global__ void __launch_bounds__(kThreads)
-mdnorm_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ MatBlock mb) {
+mdnorm_cull_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ MatBlock mb) {
   extern __shared__ double smem[];
   double* sM = smem;
   double* sC = sM + 9 * mb.nmat;
-  double* sK = sC + mb.nmat;
-  double* sF = sK + (kSmemFlux ? p.nflux : 0);
   stage_mdnorm_mats(mb, sM, sC);
-  if (kSmemFlux)
-    for (int i = threadIdx.x; i < p.nflux; i += blockDim.x) {
-      sK[i] = p.flux_k[i];
-      sF[i] = p.flux_F[i];
-    }
   __syncthreads();
-  const FluxView fx{kSmemFlux ? sK : p.flux_k, kSmemFlux ? sF : p.flux_F, p.nflux};
-  AtomicEmit emit{p.norm};
-  unsigned long long c_traj = 0, c_hit = 0, c_cross = 0, c_seg = 0;
-  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < p.nshard; i += stride) {
-    const double4 px = p.pix[p.pix_begin + i * p.pix_stride];
-    if (kStats) c_traj += mb.nmat;
-    if (px.w == 0.0) continue;  // masked pixel contributes 0 (reading #16)
-    for (int m = 0; m < mb.nmat; ++m) {
-      const double* M = sM + 9 * m;
-      double v[3] = {row_dot(M, px.x, px.y, px.z), row_dot(M + 3, px.x, px.y, px.z),
-                     row_dot(M + 6, px.x, px.y, px.z)};
-      double kin, kout;
-      if (!traj_clip(p.g, v, p.kmin, p.kmax, kin, kout)) continue;
-      int nc;
-      const int ns = traj_walk(p.g, fx, v, kin, kout, dmul(px.w, sC[m]), emit, &nc);
-      if (kStats) {
-        c_hit += 1;
-        c_cross += nc - 2;
-        c_seg += ns;
+  const int lane = threadIdx.x & 31;
+  const uint32_t nshard = (uint32_t)p.nshard;
+  unsigned long long c_traj = 0, c_hit = 0, c_cross = 0;
+  const uint32_t stride = gridDim.x * blockDim.x;
+  // warp-uniform loop so that the ballot below always has the full warp
+  for (uint32_t base = blockIdx.x * blockDim.x + (threadIdx.x & ~31u); base < p.tlen; base += stride) {
+    const uint32_t off = base + lane;
+    bool hit = false;
+    Hitter h;
+    if (off < p.tlen) {
+      const uint32_t t = p.t0 + off;
+      const uint32_t m = t / nshard;
+      const uint32_t i = t - m * nshard;
+      const double4 px = p.pix[p.pix_begin + (int64_t)i * p.pix_stride];
+      if (kStats) c_traj += 1;
+      if (px.w != 0.0) {  // masked pixels contribute 0 (reading #16)
+        const double* M = sM + 9 * m;
+        const double v0 = row_dot(M, px.x, px.y, px.z);
+        const double v1 = row_dot(M + 3, px.x, px.y, px.z);
+        const double v2 = row_dot(M + 6, px.x, px.y, px.z);
+        const double vv[3] = {v0, v1, v2};
+        double kin, kout;
+        if (traj_clip(p.g, vv, p.kmin, p.kmax, kin, kout)) {
+          hit = true;
+          AxisCursor c0, c1, c2;
+          cursor_init(c0, p.g, 0, v0, kin, kout);
+          cursor_init(c1, p.g, 1, v1, kin, kout);
+          cursor_init(c2, p.g, 2, v2, kin, kout);
+          const int total = c0.cnt + c1.cnt + c2.cnt;
+          // piece plan: cut at crossings of the busiest axis A, ~kPieceSegs segments per piece
+          int A = 0, cA = c0.cnt, jA = c0.j, sA = c0.step;
+          if (c1.cnt > cA) { A = 1; cA = c1.cnt; jA = c1.j; sA = c1.step; }
+          if (c2.cnt > cA) { A = 2; cA = c2.cnt; jA = c2.j; sA = c2.step; }
+          int P = 1, G = 1;
+          if (total + 1 > kPieceSegs && cA > 1) {
+            const int want = (total + kPieceSegs) / kPieceSegs;   // ceil((total+1)/target)
+            G = max(1, (cA + want - 1) / want);
+            P = (cA + G - 1) / G;
+          }
+          h.v0 = v0; h.v1 = v1; h.v2 = v2; h.kin = kin; h.kout = kout;
+          h.oc = dmul(px.w, sC[m]);
+          h.A = A; h.jA = jA; h.stepG = sA * G; h.P = P;
+          if (kStats) {
+            c_hit += 1;
+            c_cross += total;
+          }
+        }
+      }
+    }
+    const unsigned ballot = __ballot_sync(kFull, hit);
+    if (ballot) {
+      unsigned idx = 0;
+      if (lane == 0) idx = atomicAdd(&p.ctr->nhit, (unsigned)__popc(ballot));
+      idx = __shfl_sync(kFull, idx, 0);
+      if (hit) {
+        Hitter* dst = p.hit + idx + __popc(ballot & ((1u << lane) - 1u));
+        *dst = h;
       }
     }
   }
@@ -94,8 +134,75 @@ mdnorm_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ MatBl
     flush_counter(p.stats + 0, c_traj);
     flush_counter(p.stats + 1, c_hit);
     flush_counter(p.stats + 2, c_cross);
-    flush_counter(p.stats + 3, c_seg);
   }
+}
+
+// ---------------------------------------------------------------- M3-M7: balanced piece walk
+template <bool kSmemFlux, bool kStats>
+__global__ void __launch_bounds__(kWalkThreads)
+mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
+  extern __shared__ double2 wsm[];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int nwarps = blockDim.x >> 5;
+  double2* sKF = wsm;
+  int* sTab = reinterpret_cast<int*>(sKF + (kSmemFlux ? p.flux.n : 0));
+  int* sPre = sTab + (kSmemFlux ? p.flux.ntab : 0);
+  if (kSmemFlux) {
+    for (int i = threadIdx.x; i < p.flux.n; i += blockDim.x) sKF[i] = p.flux.kf[i];
+    for (int i = threadIdx.x; i < p.flux.ntab; i += blockDim.x) sTab[i] = p.flux.tab[i];
+  }
+  __syncthreads();
+  FluxView fx = p.flux;
+  if (kSmemFlux) {
+    fx.kf = sKF;
+    fx.tab = sTab;
+  }
+  int* pre = sPre + 32 * warp;
+  (void)nwarps;
+  AtomicEmit emit{p.norm};
+  const unsigned nhit = *(volatile unsigned*)&p.ctr->nhit;
+  unsigned long long c_seg = 0;
+  for (;;) {
+    unsigned b = 0;
+    if (lane == 0) b = atomicAdd(&p.ctr->batch, 1u);
+    b = __shfl_sync(kFull, b, 0);
+    const unsigned h0 = b * 32u;
+    if (h0 >= nhit) break;
+    const unsigned hl = h0 + lane;
+    int P = hl < nhit ? p.hit[hl].P : 0;
+    // inclusive warp scan of piece counts
+    int incl = P;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int y = __shfl_up_sync(kFull, incl, o);
+      if (lane >= o) incl += y;
+    }
+    pre[lane] = incl;
+    const int total = __shfl_sync(kFull, incl, 31);
+    __syncwarp();
+    for (int q = lane; q < total; q += 32) {
+      // owner hitter: first l with pre[l] > q
+      int l = 0;
+#pragma unroll
+      for (int s = 16; s > 0; s >>= 1)
+        if (pre[l + s - 1] <= q) l += s;
+      const int pi = q - (l ? pre[l - 1] : 0);
+      const Hitter& h = p.hit[h0 + l];
+      const double v0 = h.v0, v1 = h.v1, v2 = h.v2;
+      double lo_k = h.kin, hi_k = h.kout;
+      if (h.P > 1) {
+        const double vA = h.A == 0 ? v0 : (h.A == 1 ? v1 : v2);
+        const double rA = ddiv(1.0, vA);
+        if (pi > 0) lo_k = plane_k(p.g, h.A, h.jA + pi * h.stepG, rA);
+        if (pi < h.P - 1) hi_k = plane_k(p.g, h.A, h.jA + (pi + 1) * h.stepG, rA);
+      }
+      int nc;
+      const int ns = traj_walk(p.g, fx, v0, v1, v2, lo_k, hi_k, h.oc, emit, &nc);
+      if (kStats) c_seg += ns;
+    }
+    __syncwarp();
+  }
+  if (kStats) flush_counter(p.stats + 3, c_seg);
 }
 
 // ---------------------------------------------------------------- B1-B3: one thread per event
@@ -146,13 +253,32 @@ xs_kernel(const double* __restrict__ norm, const double* __restrict__ binmd, dou
   }
 }
 
-// ---------------------------------------------------------------- instrument table (M1 q_p)
+// ---------------------------------------------------------------- setup kernels
 __global__ void pixels_prepare_kernel(const double* __restrict__ dir, const double* __restrict__ solid,
                                       double4* __restrict__ pix, int64_t npix) {
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < npix; i += stride) {
     // q_p = z - d_p (reading #1): (-d_x, -d_y, 1 - d_z)
     pix[i] = make_double4(-dir[3 * i], -dir[3 * i + 1], dsub(1.0, dir[3 * i + 2]), solid[i]);
+  }
+}
+
+// tab[c] = max{i : kappa_i <= kappa_0 + c * cell}: a start index for the flux search (M5)
+__global__ void flux_table_kernel(const double2* __restrict__ kf, int n, int* __restrict__ tab, int ntab,
+                                  double k0, double cell) {
+  for (int c = blockIdx.x * blockDim.x + threadIdx.x; c < ntab; c += gridDim.x * blockDim.x) {
+    const double x = k0 + (double)c * cell;
+    int lo = 0, hi = n - 1;
+    if (x >= kf[n - 1].x) {
+      tab[c] = n - 2;
+      continue;
+    }
+    while (hi - lo > 1) {
+      const int mid = (lo + hi) >> 1;
+      if (kf[mid].x <= x) lo = mid;
+      else hi = mid;
+    }
+    tab[c] = lo;
   }
 }
 
@@ -186,19 +312,18 @@ debug_traj_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ M
   const int64_t pi = id - (int64_t)m * npix;
   const double4 px = p.pix[pi];
   const double* M = sM + 9 * m;
-  double v[3] = {row_dot(M, px.x, px.y, px.z), row_dot(M + 3, px.x, px.y, px.z),
-                 row_dot(M + 6, px.x, px.y, px.z)};
+  const double v[3] = {row_dot(M, px.x, px.y, px.z), row_dot(M + 3, px.x, px.y, px.z),
+                       row_dot(M + 6, px.x, px.y, px.z)};
   double kin, kout;
   if (!traj_clip(p.g, v, p.kmin, p.kmax, kin, kout)) {
     n_cross[t] = 0;
     n_seg[t] = 0;
     return;
   }
-  const FluxView fx{p.flux_k, p.flux_F, p.nflux};
   RecordEmit rec{seg_bins + t * max_segs, seg_vals + t * max_segs, max_segs, 0};
   int nc;
-  n_seg[t] = traj_walk(p.g, fx, v, kin, kout, dmul(px.w, sC[m]), rec, &nc);
-  n_cross[t] = nc;
+  n_seg[t] = traj_walk(p.g, p.flux, v[0], v[1], v[2], kin, kout, dmul(px.w, sC[m]), rec, &nc);
+  n_cross[t] = nc + 2;  // |L| = clip endpoints + crossings
 }
 
 __global__ void __launch_bounds__(kThreads)
@@ -229,10 +354,34 @@ __global__ void debug_compose_kernel(const __grid_constant__ MatBlock mdn,
     if (!compose_binmd(bin.UB, bin.u.c.ops + 9 * m, bin.W, N + 9 * m)) ok[0] = 0;
 }
 
-int grid_for(int64_t work, int num_sms, int per_sm) {
-  int64_t blocks = (work + kThreads - 1) / kThreads;
+int grid_for(int64_t work, int num_sms, int per_sm, int threads = kThreads) {
+  int64_t blocks = (work + threads - 1) / threads;
   blocks = std::min<int64_t>(blocks, (int64_t)num_sms * per_sm);
   return (int)std::max<int64_t>(blocks, 1);
+}
+
+template <bool kSmemFlux, bool kStats>
+cudaError_t launch_walk(const MdnParams& p, int num_sms, cudaStream_t s) {
+  const size_t smem = (kSmemFlux ? sizeof(double2) * p.flux.n + sizeof(int) * p.flux.ntab : 0) +
+                      sizeof(int) * 32 * (kWalkThreads / 32);
+  auto k = mdnorm_walk_kernel<kSmemFlux, kStats>;
+  cudaError_t err = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (err != cudaSuccess) return err;
+  int per_sm = 0;
+  err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kWalkThreads, smem);
+  if (err != cudaSuccess) return err;
+  k<<<num_sms * std::max(per_sm, 1), kWalkThreads, smem, s>>>(p);
+  return cudaGetLastError();
+}
+
+template <bool kStats>
+cudaError_t launch_cull(const MdnParams& p, const MatBlock& mb, int num_sms, cudaStream_t s) {
+  const size_t smem = sizeof(double) * 10 * (size_t)mb.nmat;
+  auto k = mdnorm_cull_kernel<kStats>;
+  cudaError_t err = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (err != cudaSuccess) return err;
+  k<<<grid_for(p.tlen, num_sms, 16), kThreads, smem, s>>>(p, mb);
+  return cudaGetLastError();
 }
 
 }  // namespace
@@ -243,24 +392,22 @@ cudaError_t launch_pixels_prepare(const double* dir, const double* solid, double
   return cudaGetLastError();
 }
 
-template <bool kSmemFlux, bool kStats>
-cudaError_t launch_mdnorm_t(const MdnParams& p, const MatBlock& mb, int num_sms, size_t smem, cudaStream_t s) {
-  cudaError_t err = cudaFuncSetAttribute(mdnorm_kernel<kSmemFlux, kStats>,
-                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  if (err != cudaSuccess) return err;
-  mdnorm_kernel<kSmemFlux, kStats><<<grid_for(p.nshard, num_sms, 8), kThreads, smem, s>>>(p, mb);
+cudaError_t launch_flux_table(const double2* kf, int n, int* tab, int ntab, double k0, double cell,
+                              cudaStream_t s) {
+  flux_table_kernel<<<grid_for(ntab, 148, 8), kThreads, 0, s>>>(kf, n, tab, ntab, k0, cell);
   return cudaGetLastError();
 }
 
 cudaError_t launch_mdnorm(const MdnParams& p, const MatBlock& mb, int num_sms, cudaStream_t s) {
-  if (p.nshard <= 0 || mb.nmat <= 0) return cudaSuccess;
-  const bool smem_flux = p.nflux <= kFluxSmemMax;
-  const size_t smem = sizeof(double) * (10 * (size_t)mb.nmat + (smem_flux ? 2 * (size_t)p.nflux : 0));
+  if (p.tlen == 0 || mb.nmat <= 0) return cudaSuccess;
+  cudaError_t err = cudaMemsetAsync(p.ctr, 0, sizeof(DevCounters), s);
+  if (err != cudaSuccess) return err;
+  err = p.stats ? launch_cull<true>(p, mb, num_sms, s) : launch_cull<false>(p, mb, num_sms, s);
+  if (err != cudaSuccess) return err;
+  const bool smem_flux = p.flux.n <= kFluxSmemMax;
   if (smem_flux)
-    return p.stats ? launch_mdnorm_t<true, true>(p, mb, num_sms, smem, s)
-                   : launch_mdnorm_t<true, false>(p, mb, num_sms, smem, s);
-  return p.stats ? launch_mdnorm_t<false, true>(p, mb, num_sms, smem, s)
-                 : launch_mdnorm_t<false, false>(p, mb, num_sms, smem, s);
+    return p.stats ? launch_walk<true, true>(p, num_sms, s) : launch_walk<true, false>(p, num_sms, s);
+  return p.stats ? launch_walk<false, true>(p, num_sms, s) : launch_walk<false, false>(p, num_sms, s);
 }
 
 cudaError_t launch_binmd(const BinParams& p, const MatBlock& mb, int num_sms, cudaStream_t s) {

@@ -10,7 +10,8 @@ namespace mdn {
 constexpr int kMaxOps = 48;           // MDN_MAX_OPS
 constexpr int kMaxMats = 64;          // MDN_MAX_MATS
 constexpr int kRunsPerLaunch = 16;    // runs composed per MDNorm launch (batched API)
-constexpr int kFluxSmemMax = 4096;    // flux knots staged in shared memory (64 KB fp64 pairs)
+constexpr int kFluxSmemMax = 4096;    // flux knots staged in shared memory (64 KB of double2)
+constexpr int kPieceSegs = 24;        // target segments per work piece (load balance, M4-M7)
 
 // Matrices for one launch, passed by value as a __grid_constant__ kernel parameter (sm_70+
 // kernels accept up to 32 KB of parameters; CUDA >= 12.1).  Either compose (UB, W, ops, R) on
@@ -32,17 +33,34 @@ struct MatBlock {
   } u;
 };
 
+// A trajectory that hits the grid (output of the cull kernel, input of the walk kernel): its
+// direction v, clip [kin, kout], weight Omega_p c_r, and how it is cut into P pieces at the
+// crossings of axis A with indices j_A + p * stepG (p = 1 .. P-1).
+struct alignas(16) Hitter {
+  double v0, v1, v2, kin;
+  double kout, oc;
+  int32_t A, jA, stepG, P;
+};
+
+struct DevCounters {
+  unsigned int nhit;     // hitters written by the cull kernel
+  unsigned int batch;    // warp batches claimed by the walk kernel
+  unsigned int pad[2];
+};
+
 struct MdnParams {
   GridC g;
   const double4* pix;      // (q0, q1, q2, Omega) per pixel, q = z - d  (M1)
   int64_t pix_begin, pix_stride, nshard;
-  const double* flux_k;
-  const double* flux_F;
-  int32_t nflux;
+  FluxView flux;           // device pointers (global)
   int32_t acc_f32;
   double kmin, kmax;
   double* norm;            // fp64 histogram (nbins)
   unsigned long long* stats;  // nullptr, or [traj, hits, crossings, segments] (+= per launch)
+  // cull -> walk hand-off (production path)
+  Hitter* hit;             // capacity >= slab length
+  DevCounters* ctr;
+  uint32_t t0, tlen;       // slab of trajectory indices t = m * nshard + i
 };
 
 struct BinParams {
@@ -52,12 +70,15 @@ struct BinParams {
   int32_t col_w, col_q;
   int32_t acc_f32;
   double* binmd;           // fp64 histogram (nbins)
-  unsigned long long* stats;  // nullptr, or [pairs, inside] (+= per launch)
+  unsigned long long* stats;  // nullptr, or [.., .., .., .., pairs, inside] (+= per launch)
 };
 
 // launchers (return the launch's cudaError_t)
 cudaError_t launch_pixels_prepare(const double* dir, const double* solid, double4* pix, int64_t npix,
                                   cudaStream_t s);
+cudaError_t launch_flux_table(const double2* kf, int n, int* tab, int ntab, double k0, double cell,
+                              cudaStream_t s);
+// MDNorm for trajectories [p.t0, p.t0 + p.tlen): cull (M1-M3) + piece walk (M3-M7).
 cudaError_t launch_mdnorm(const MdnParams& p, const MatBlock& mb, int num_sms, cudaStream_t s);
 cudaError_t launch_binmd(const BinParams& p, const MatBlock& mb, int num_sms, cudaStream_t s);
 cudaError_t launch_cross_section(const double* norm, const double* binmd, double* xs, int64_t nbins,
