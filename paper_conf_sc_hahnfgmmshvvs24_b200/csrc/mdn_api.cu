@@ -3,6 +3,7 @@
 // Host side only: argument validation (before any side effect), device-memory ownership,
 // stream ordering and launch marshalling.  Every step of the hot path itself (matrix
 // composition, trajectories, scatter, divide) runs in the kernels of mdn_kernels.cu.
+#include <algorithm>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
@@ -29,6 +30,7 @@ struct mdn_grid {
   int* d_ftab = nullptr;      // flux search start table (nftab cells)
   int32_t nflux = 0, nftab = 0;
   double ftab_k0 = 0.0, ftab_inv_cell = 0.0;
+  int ftab_nsteps = 0;
   mdn::Hitter* d_hit = nullptr;       // cull -> walk hand-off buffer
   uint32_t hit_cap = 0;
   mdn::DevCounters* d_ctr = nullptr;
@@ -174,6 +176,7 @@ mdn::MdnParams mdn_params(mdn_grid* g, double k_min, double k_max, int64_t pix_b
   p.flux.inv_cell = g->ftab_inv_cell;
   p.flux.n = g->nflux;
   p.flux.ntab = g->nftab;
+  p.flux.nsteps = g->ftab_nsteps;
   p.acc_f32 = g->acc == MDN_ACC_F32;
   p.kmin = k_min;
   p.kmax = k_max;
@@ -193,7 +196,6 @@ constexpr uint32_t kMaxSlab = 1u << 24;  // trajectories per cull/walk pair (1 G
 mdn_status run_mdnorm(mdn_grid* g, mdn::MdnParams p, const MatBlock& mb, cudaStream_t s) {
   const uint64_t ntraj = (uint64_t)mb.nmat * (uint64_t)p.nshard;
   if (ntraj == 0) return MDN_OK;
-  if (ntraj >= (1ull << 32)) return fail(MDN_EINVAL, "too many trajectories in one launch (%llu)", (unsigned long long)ntraj);
   const uint32_t want = (uint32_t)std::min<uint64_t>(ntraj, kMaxSlab);
   if (g->hit_cap < want) {
     if (g->d_hit) {
@@ -208,9 +210,11 @@ mdn_status run_mdnorm(mdn_grid* g, mdn::MdnParams p, const MatBlock& mb, cudaStr
   if (!g->d_ctr) MDN_CUDA(cudaMalloc(&g->d_ctr, sizeof(mdn::DevCounters)), "counters");
   p.hit = g->d_hit;
   p.ctr = g->d_ctr;
-  for (uint64_t t0 = 0; t0 < ntraj; t0 += g->hit_cap) {
-    p.t0 = (uint32_t)t0;
-    p.tlen = (uint32_t)std::min<uint64_t>(g->hit_cap, ntraj - t0);
+  // pixels per slab so that every trajectory of the slab can be a hitter
+  const uint64_t per = std::max<uint64_t>(1, g->hit_cap / (uint64_t)mb.nmat);
+  for (uint64_t p0 = 0; p0 < (uint64_t)p.nshard; p0 += per) {
+    p.p0 = (uint32_t)p0;
+    p.plen = (uint32_t)std::min<uint64_t>(per, (uint64_t)p.nshard - p0);
     MDN_CUDA(mdn::launch_mdnorm(p, mb, g->num_sms, s), "mdnorm kernels");
   }
   return MDN_OK;
@@ -233,6 +237,10 @@ mdn::BinParams bin_params(mdn_grid* g, const float* ev, int64_t n, int64_t strid
   p.stride = stride;
   p.col_w = col_w;
   p.col_q = col_q;
+  // fp32 fast-path axis order: fewest bins first (stable), so a thin slab axis rejects early
+  int ord[3] = {0, 1, 2};
+  std::stable_sort(ord, ord + 3, [&](int a, int b) { return g->g.n[a] < g->g.n[b]; });
+  for (int a = 0; a < 3; ++a) p.ord[a] = ord[a];
   p.acc_f32 = g->acc == MDN_ACC_F32;
   p.binmd = g->d_hist + g->g.nbins;
   p.stats = g->stats_on ? g->d_stats : nullptr;
@@ -312,7 +320,7 @@ mdn_status mdnorm_create_grid(int device, const double lo[3], const double hi[3]
       return fail(MDN_EINVAL, "axis %d: need finite lo < hi (got %g, %g)", a, lo[a], hi[a]);
     if (nbins[a] < 1 || nbins[a] > (1ll << 30)) return fail(MDN_EINVAL, "axis %d: nbins %lld outside [1, 2^30]", a, (long long)nbins[a]);
     total *= nbins[a];
-    if (total > (1ll << 40)) return fail(MDN_EINVAL, "grid too large");
+    if (total >= (1ll << 31)) return fail(MDN_EINVAL, "grid too large (at most 2^31 - 1 bins)");
   }
   if (!finite_all(W, 9) || !nonsingular(W)) return fail(MDN_EINVAL, "W is singular or non-finite");
   if (acc != MDN_ACC_F64 && acc != MDN_ACC_F32) return fail(MDN_EINVAL, "unknown accumulation mode %d", (int)acc);
@@ -417,13 +425,28 @@ mdn_status mdnorm_set_flux(mdn_grid* g, int64_t n, const double* k, const double
   for (int64_t i = 0; i < n; ++i) kf[i] = make_double2(hk[i], hF[i]);
   const int ntab = (int)std::min<int64_t>(2 * n, 1 << 22);
   const double cell = (hk[n - 1] - hk[0]) / (double)ntab;
+  // tab[c] = max{i : kappa_i <= fl(kappa_0 + c * cell)} (exact comparisons); the search window
+  // of a query in cell c is [tab[c-1], tab[c+2] + 1] (flux_at), nsteps bisections close it
+  std::vector<int> htab((size_t)ntab);
+  for (int c = 0, i = 0; c < ntab; ++c) {
+    const double x = hk[0] + (double)c * cell;
+    while (i + 1 < n - 1 && hk[i + 1] <= x) ++i;
+    htab[c] = i;
+  }
+  int wmax = 1;
+  for (int c = 0; c < ntab; ++c) {
+    const int lo = htab[std::max(c - 1, 0)];
+    const int hi = c + 2 < ntab ? htab[c + 2] + 1 : (int)n - 1;
+    wmax = std::max(wmax, hi - lo);
+  }
+  int nsteps = 0;
+  while ((1 << nsteps) < wmax) ++nsteps;
   double2* d = nullptr;
   int* tab = nullptr;
   cudaError_t e = cudaMalloc(&d, sizeof(double2) * n);
   if (e == cudaSuccess) e = cudaMalloc(&tab, sizeof(int) * ntab);
   if (e == cudaSuccess) e = cudaMemcpy(d, kf.data(), sizeof(double2) * n, cudaMemcpyHostToDevice);
-  if (e == cudaSuccess) e = mdn::launch_flux_table(d, (int)n, tab, ntab, hk[0], cell, nullptr);
-  if (e == cudaSuccess) e = cudaDeviceSynchronize();
+  if (e == cudaSuccess) e = cudaMemcpy(tab, htab.data(), sizeof(int) * ntab, cudaMemcpyHostToDevice);
   if (e != cudaSuccess) {
     cudaFree(d);
     cudaFree(tab);
@@ -437,6 +460,7 @@ mdn_status mdnorm_set_flux(mdn_grid* g, int64_t n, const double* k, const double
   g->nftab = ntab;
   g->ftab_k0 = hk[0];
   g->ftab_inv_cell = 1.0 / cell;
+  g->ftab_nsteps = nsteps;
   return ok();
 }
 

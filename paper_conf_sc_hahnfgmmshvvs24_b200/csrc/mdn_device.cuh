@@ -94,32 +94,43 @@ __device__ __forceinline__ bool compose_binmd(const double* UB, const double* S,
 // ------------------------------------------------------------------------------ M5 flux
 // F(x): clamp outside, else i = max{i : kappa_i <= x} and
 //   Phi_i + (Phi_{i+1} - Phi_i) * ((x - kappa_i) / (kappa_{i+1} - kappa_i)).
-// i is unique, so it may be found by any search: here a uniform-cell index table gives a start
-// index that is then corrected by exact comparisons (O(1) expected instead of a 12-step binary
-// search).  tab[c] = max{i : kappa_i <= kappa_0 + c * cell} (setup kernel; any monotone guess
-// would do because the loops below fix it).
+// i is unique, so it may be found by any search.  Here a uniform-cell table narrows it to a
+// window: tab[c] = max{i : kappa_i <= fl(kappa_0 + c * cell)} (host, exact comparisons).  The
+// cell c of x is computed approximately (off by at most one cell), so the window
+// [tab[c-1], tab[c+2] + 1] always satisfies kappa_lo <= x < kappa_hi; a fixed number of
+// branch-free bisection steps (nsteps = ceil(log2(max window)), warp-uniform) then lands on i.
 struct FluxView {
   const double2* kf;  // (kappa_i, Phi_i)
   const int* tab;     // ntab cell start indices
   double k0, inv_cell;
-  int n, ntab;
+  int n, ntab, nsteps, pad;
 };
 
 __device__ __forceinline__ double flux_at(const FluxView& f, double x) {
   const double2 first = f.kf[0], last = f.kf[f.n - 1];
   if (x <= first.x) return first.y;
   if (x >= last.x) return last.y;
-  double u = (x - first.x) * f.inv_cell;  // any rounding: only a starting guess
-  int c = u < (double)f.ntab ? (int)u : f.ntab - 1;
-  int i = f.tab[c < 0 ? 0 : c];
-  while (i > 0 && f.kf[i].x > x) --i;
-  double2 lo = f.kf[i], hi = f.kf[i + 1];
-  while (hi.x <= x) {  // terminates: x < kappa_{n-1}
-    ++i;
-    lo = hi;
-    hi = f.kf[i + 1];
+  const double u = (x - first.x) * f.inv_cell;  // any rounding: only selects the window
+  const int c = u < (double)(f.ntab - 1) ? (int)u : f.ntab - 1;
+  int lo = f.tab[max(c - 1, 0)];
+  int hi = c + 2 < f.ntab ? f.tab[c + 2] + 1 : f.n - 1;
+#pragma unroll
+  for (int s = 0; s < 4; ++s) {  // invariant kappa_lo <= x < kappa_hi (nsteps is warp-uniform)
+    if (s < f.nsteps) {
+      const int mid = (lo + hi) >> 1;
+      const bool le = f.kf[mid].x <= x;
+      lo = le ? mid : lo;
+      hi = le ? hi : mid;
+    }
   }
-  return dadd(lo.y, dmul(dsub(hi.y, lo.y), ddiv(dsub(x, lo.x), dsub(hi.x, lo.x))));
+  for (int s = 4; s < f.nsteps; ++s) {  // only for very uneven knot spacing
+    const int mid = (lo + hi) >> 1;
+    const bool le = f.kf[mid].x <= x;
+    lo = le ? mid : lo;
+    hi = le ? hi : mid;
+  }
+  const double2 a = f.kf[lo], b = f.kf[lo + 1];
+  return dadd(a.y, dmul(dsub(b.y, a.y), ddiv(dsub(x, a.x), dsub(b.x, a.x))));
 }
 
 // ------------------------------------------------------------------------------ M1-M2
@@ -210,26 +221,21 @@ __device__ __forceinline__ AxisStream axis_stream(const GridC& g, int a, double 
   return s;
 }
 
-// One axis of the merge: reciprocal, position in its stream, next crossing value.
+// One axis of the merge: reciprocal, position (j kept as an exact double so that the edge
+// lo + j * w needs no int->double conversion), remaining count, next crossing value.
 struct AxisCursor {
-  double r, nk;
-  int j, cnt, step;
+  double r, nk, jd, stepd;
+  int cnt;
 };
 
 __device__ __forceinline__ void cursor_init(AxisCursor& c, const GridC& g, int a, double v, double lo_k,
                                             double hi_k) {
   c.r = v != 0.0 ? ddiv(1.0, v) : 0.0;
   const AxisStream s = axis_stream(g, a, v, c.r, lo_k, hi_k);
-  c.j = s.j;
+  c.jd = (double)s.j;
+  c.stepd = (double)s.step;
   c.cnt = s.cnt;
-  c.step = s.step;
-  c.nk = s.cnt > 0 ? plane_k(g, a, s.j, c.r) : CUDART_INF;
-}
-
-__device__ __forceinline__ void cursor_advance(AxisCursor& c, const GridC& g, int a) {
-  c.cnt -= 1;
-  c.j += c.step;
-  c.nk = c.cnt > 0 ? plane_k(g, a, c.j, c.r) : CUDART_INF;
+  c.nk = s.cnt > 0 ? dmul(dadd(g.lo[a], dmul(c.jd, g.w[a])), c.r) : CUDART_INF;
 }
 
 // ------------------------------------------------------------------------------ M4-M7
@@ -239,33 +245,47 @@ __device__ __forceinline__ void cursor_advance(AxisCursor& c, const GridC& g, in
 // P:115, and the GPU comb sort, with no buffer), flux at each list entry (M5), midpoint
 // bin of every positive-length segment (M6) and emit(b, (F(k2) - F(k1)) * omega_c) (M7).
 // Splitting L at any of its members leaves the set of segments unchanged, which is what lets
-// the production kernel cut long trajectories into balanced pieces.  Returns n_seg; *ncross
-// receives the number of crossings strictly inside (lo_k, hi_k).
-template <class Emit>
+// the production kernel cut long trajectories into balanced pieces.  The merge step is written
+// with selects only (no per-axis branches) so that the lanes of a warp stay converged.
+// Returns n_seg; *ncross receives the number of crossings strictly inside (lo_k, hi_k).
+template <bool k3D, class Emit>
 __device__ __forceinline__ int traj_walk(const GridC& g, const FluxView& fx, double v0, double v1,
                                          double v2, double lo_k, double hi_k, double omega_c,
                                          Emit& emit, int* ncross) {
+  // k3D = false: the last axis has a single bin (2-D slice), so it never has a crossing
   AxisCursor c0, c1, c2;
   cursor_init(c0, g, 0, v0, lo_k, hi_k);
   cursor_init(c1, g, 1, v1, lo_k, hi_k);
-  cursor_init(c2, g, 2, v2, lo_k, hi_k);
+  if (k3D) {
+    cursor_init(c2, g, 2, v2, lo_k, hi_k);
+  } else {
+    c2.cnt = 0;
+    c2.nk = CUDART_INF;
+    c2.jd = c2.stepd = c2.r = 0.0;
+  }
   const int total = c0.cnt + c1.cnt + c2.cnt;
   *ncross = total;
   double k1 = lo_k, F1 = flux_at(fx, lo_k);
   int nseg = 0;
-  for (int left = total;; --left) {
-    double k2;
+  for (int left = total; left >= 0; --left) {
+    // smallest pending crossing (ties: lowest axis first; equal values give a skipped
+    // zero-length segment, so the order among ties never matters)
+    const bool s01 = c1.nk < c0.nk;
+    const double m01 = s01 ? c1.nk : c0.nk;
+    const bool s2 = k3D && c2.nk < m01;
+    const bool p0 = !s2 && !s01, p1 = !s2 && s01;
+    double k2 = s2 ? c2.nk : m01;
+    // advance the chosen axis (selects, one plane evaluation)
+    const double jd = (p0 ? c0.jd + c0.stepd : (p1 ? c1.jd + c1.stepd : c2.jd + c2.stepd));
+    const int cnt = (p0 ? c0.cnt : (p1 ? c1.cnt : c2.cnt)) - 1;
+    const double lo = p0 ? g.lo[0] : (p1 ? g.lo[1] : g.lo[2]);
+    const double w = p0 ? g.w[0] : (p1 ? g.w[1] : g.w[2]);
+    const double r = p0 ? c0.r : (p1 ? c1.r : c2.r);
+    const double nk = cnt > 0 ? dmul(dadd(lo, dmul(jd, w)), r) : CUDART_INF;
     if (left > 0) {
-      if (c0.nk <= c1.nk && c0.nk <= c2.nk) {
-        k2 = c0.nk;
-        cursor_advance(c0, g, 0);
-      } else if (c1.nk <= c2.nk) {
-        k2 = c1.nk;
-        cursor_advance(c1, g, 1);
-      } else {
-        k2 = c2.nk;
-        cursor_advance(c2, g, 2);
-      }
+      if (p0) { c0.jd = jd; c0.cnt = cnt; c0.nk = nk; }
+      if (p1) { c1.jd = jd; c1.cnt = cnt; c1.nk = nk; }
+      if (k3D && s2) { c2.jd = jd; c2.cnt = cnt; c2.nk = nk; }
     } else {
       k2 = hi_k;
     }
@@ -277,16 +297,13 @@ __device__ __forceinline__ int traj_walk(const GridC& g, const FluxView& fx, dou
       const double t2 = dmul(dsub(dmul(km, v2), g.lo[2]), g.s[2]);
       if (0.0 <= t0 && t0 < (double)g.n[0] && 0.0 <= t1 && t1 < (double)g.n[1] && 0.0 <= t2 &&
           t2 < (double)g.n[2]) {
-        const int64_t b = (int64_t)__double2int_rz(t0) +
-                          (int64_t)g.n[0] * ((int64_t)__double2int_rz(t1) +
-                                             (int64_t)g.n[1] * __double2int_rz(t2));
+        const int b = __double2int_rz(t0) + g.n[0] * (__double2int_rz(t1) + g.n[1] * __double2int_rz(t2));
         emit(b, dmul(dsub(F2, F1), omega_c));
         ++nseg;
       }
       k1 = k2;
       F1 = F2;
     }
-    if (left == 0) break;
   }
   return nseg;
 }

@@ -58,34 +58,61 @@ __device__ __forceinline__ void flush_counter(unsigned long long* dst, unsigned 
 
 struct AtomicEmit {
   double* h;
-  __device__ __forceinline__ void operator()(int64_t b, double val) const { atomicAdd(h + b, val); }
+  __device__ __forceinline__ void operator()(int b, double val) const { atomicAdd(h + b, val); }
 };
 
 // ---------------------------------------------------------------- M1-M3: cull + compaction
+// One thread per pixel of the slab, looping over every (run, op) matrix of the launch (pixel
+// read once; matrices are warp-uniform smem broadcasts).  A conservative fp32 slab test with a
+// proven error margin rejects most misses without any fp64 division; every
+// survivor gets the exact fp64 v and clip, so the hit decision is the definition's.
+struct CullMat {
+  float M[9];
+  float delta[3];  // per-axis margin of the fp32 test
+};
+
 template <bool kStats>
 __global__ void __launch_bounds__(kThreads)
 mdnorm_cull_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ MatBlock mb) {
   extern __shared__ double smem[];
   double* sM = smem;
   double* sC = sM + 9 * mb.nmat;
+  CullMat* sF = reinterpret_cast<CullMat*>(sC + mb.nmat);
   stage_mdnorm_mats(mb, sM, sC);
   __syncthreads();
+  for (int m = threadIdx.x; m < mb.nmat; m += blockDim.x) {
+    for (int a = 0; a < 3; ++a) {
+      double sum = 0.0;
+      for (int i = 0; i < 3; ++i) {
+        sF[m].M[3 * a + i] = (float)sM[9 * m + 3 * a + i];
+        sum += fabs(sM[9 * m + 3 * a + i]);
+      }
+      // |q_i| <= 2; fp32 v and x = k v are within 1e-6 kmax sum|M_a| of the exact values
+      sF[m].delta[a] = (float)(4e-6 * p.kmax * sum + 1e-6 * (fabs(p.g.lo[a]) + fabs(p.g.hi[a])) + 1e-30);
+    }
+  }
+  __syncthreads();
+  const float kmin32 = (float)p.kmin, kmax32 = (float)p.kmax;
+  const float lo32[3] = {(float)p.g.lo[0], (float)p.g.lo[1], (float)p.g.lo[2]};
+  const float hi32[3] = {(float)p.g.hi[0], (float)p.g.hi[1], (float)p.g.hi[2]};
   const int lane = threadIdx.x & 31;
-  const uint32_t nshard = (uint32_t)p.nshard;
+  // per-warp ring of fp32 survivors (pixel offset, matrix); the exact fp64 path runs only when
+  // 32 of them are queued, so it executes with the whole warp converged
+  uint32_t* qoff = reinterpret_cast<uint32_t*>(sF + mb.nmat) + (threadIdx.x >> 5) * 128;
+  uint32_t* qmat = qoff + 64;
+  int qhead = 0, qcnt = 0;
   unsigned long long c_traj = 0, c_hit = 0, c_cross = 0;
-  const uint32_t stride = gridDim.x * blockDim.x;
-  // warp-uniform loop so that the ballot below always has the full warp
-  for (uint32_t base = blockIdx.x * blockDim.x + (threadIdx.x & ~31u); base < p.tlen; base += stride) {
-    const uint32_t off = base + lane;
+
+  // exact M1-M3 for queued candidates [qhead, qhead + n) (n <= 32), hitters appended
+  auto drain = [&](int n) {
+    __syncwarp();
     bool hit = false;
     Hitter h;
-    if (off < p.tlen) {
-      const uint32_t t = p.t0 + off;
-      const uint32_t m = t / nshard;
-      const uint32_t i = t - m * nshard;
-      const double4 px = p.pix[p.pix_begin + (int64_t)i * p.pix_stride];
-      if (kStats) c_traj += 1;
-      if (px.w != 0.0) {  // masked pixels contribute 0 (reading #16)
+    if (lane < n) {
+      const int slot = (qhead + lane) & 63;
+      const uint32_t off = qoff[slot], m = qmat[slot];
+      const double4 px = p.pix[p.pix_begin + (int64_t)(p.p0 + off) * p.pix_stride];
+      {
         const double* M = sM + 9 * m;
         const double v0 = row_dot(M, px.x, px.y, px.z);
         const double v1 = row_dot(M + 3, px.x, px.y, px.z);
@@ -94,24 +121,25 @@ mdnorm_cull_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ 
         double kin, kout;
         if (traj_clip(p.g, vv, p.kmin, p.kmax, kin, kout)) {
           hit = true;
-          AxisCursor c0, c1, c2;
-          cursor_init(c0, p.g, 0, v0, kin, kout);
-          cursor_init(c1, p.g, 1, v1, kin, kout);
-          cursor_init(c2, p.g, 2, v2, kin, kout);
-          const int total = c0.cnt + c1.cnt + c2.cnt;
+          const AxisStream s0 = axis_stream(p.g, 0, v0, v0 != 0.0 ? ddiv(1.0, v0) : 0.0, kin, kout);
+          const AxisStream s1 = axis_stream(p.g, 1, v1, v1 != 0.0 ? ddiv(1.0, v1) : 0.0, kin, kout);
+          const AxisStream s2 = axis_stream(p.g, 2, v2, v2 != 0.0 ? ddiv(1.0, v2) : 0.0, kin, kout);
+          const int total = s0.cnt + s1.cnt + s2.cnt;
           // piece plan: cut at crossings of the busiest axis A, ~kPieceSegs segments per piece
-          int A = 0, cA = c0.cnt, jA = c0.j, sA = c0.step;
-          if (c1.cnt > cA) { A = 1; cA = c1.cnt; jA = c1.j; sA = c1.step; }
-          if (c2.cnt > cA) { A = 2; cA = c2.cnt; jA = c2.j; sA = c2.step; }
+          const bool a1 = s1.cnt > s0.cnt;
+          const AxisStream s01 = a1 ? s1 : s0;
+          const bool a2 = s2.cnt > s01.cnt;
+          const AxisStream sa = a2 ? s2 : s01;
+          const int A = a2 ? 2 : (a1 ? 1 : 0);
           int P = 1, G = 1;
-          if (total + 1 > kPieceSegs && cA > 1) {
-            const int want = (total + kPieceSegs) / kPieceSegs;   // ceil((total+1)/target)
-            G = max(1, (cA + want - 1) / want);
-            P = (cA + G - 1) / G;
+          if (total + 1 > kPieceSegs && sa.cnt > 1) {
+            const int want = (total + kPieceSegs) / kPieceSegs;  // ceil((total + 1) / target)
+            G = max(1, (sa.cnt + want - 1) / want);
+            P = (sa.cnt + G - 1) / G;
           }
           h.v0 = v0; h.v1 = v1; h.v2 = v2; h.kin = kin; h.kout = kout;
           h.oc = dmul(px.w, sC[m]);
-          h.A = A; h.jA = jA; h.stepG = sA * G; h.P = P;
+          h.A = A; h.jA = sa.j; h.stepG = sa.step * G; h.P = P;
           if (kStats) {
             c_hit += 1;
             c_cross += total;
@@ -124,12 +152,44 @@ mdnorm_cull_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ 
       unsigned idx = 0;
       if (lane == 0) idx = atomicAdd(&p.ctr->nhit, (unsigned)__popc(ballot));
       idx = __shfl_sync(kFull, idx, 0);
-      if (hit) {
-        Hitter* dst = p.hit + idx + __popc(ballot & ((1u << lane) - 1u));
-        *dst = h;
+      if (hit) p.hit[idx + __popc(ballot & ((1u << lane) - 1u))] = h;
+    }
+    qhead = (qhead + n) & 63;
+    qcnt -= n;
+    __syncwarp();
+  };
+
+  const uint32_t stride = gridDim.x * blockDim.x;
+  // warp-uniform loops so that the ballots below always have the full warp
+  for (uint32_t base = blockIdx.x * blockDim.x + (threadIdx.x & ~31u); base < p.plen; base += stride) {
+    const uint32_t off = base + lane;
+    const bool valid = off < p.plen;
+    double4 px = make_double4(0.0, 0.0, 0.0, 0.0);
+    if (valid) px = p.pix[p.pix_begin + (int64_t)(p.p0 + off) * p.pix_stride];
+    if (kStats && valid) c_traj += mb.nmat;
+    const bool live = valid && px.w != 0.0;  // masked pixels contribute 0 (reading #16)
+    const float q0 = (float)px.x, q1 = (float)px.y, q2 = (float)px.z;
+    for (int m = 0; m < mb.nmat; ++m) {
+      const CullMat& cm = sF[m];
+      bool maybe = live;
+#pragma unroll
+      for (int a = 0; a < 3; ++a) {
+        const float v = fmaf(cm.M[3 * a + 2], q2, fmaf(cm.M[3 * a + 1], q1, cm.M[3 * a] * q0));
+        const float xa = kmin32 * v, xb = kmax32 * v;
+        const float xl = fminf(xa, xb), xh = fmaxf(xa, xb);
+        maybe = maybe && !(xh < lo32[a] - cm.delta[a] || xl >= hi32[a] + cm.delta[a]);
       }
+      const unsigned mask = __ballot_sync(kFull, maybe);
+      if (maybe) {
+        const int slot = (qhead + qcnt + __popc(mask & ((1u << lane) - 1u))) & 63;
+        qoff[slot] = off;
+        qmat[slot] = (uint32_t)m;
+      }
+      qcnt += __popc(mask);
+      if (qcnt >= 32) drain(32);
     }
   }
+  if (qcnt > 0) drain(qcnt);
   if (kStats) {
     flush_counter(p.stats + 0, c_traj);
     flush_counter(p.stats + 1, c_hit);
@@ -138,8 +198,8 @@ mdnorm_cull_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ 
 }
 
 // ---------------------------------------------------------------- M3-M7: balanced piece walk
-template <bool kSmemFlux, bool kStats>
-__global__ void __launch_bounds__(kWalkThreads)
+template <bool kSmemFlux, bool kStats, bool k3D>
+__global__ void __launch_bounds__(kWalkThreads, 2)
 mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
   extern __shared__ double2 wsm[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -180,37 +240,70 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
     pre[lane] = incl;
     const int total = __shfl_sync(kFull, incl, 31);
     __syncwarp();
-    for (int q = lane; q < total; q += 32) {
-      // owner hitter: first l with pre[l] > q
-      int l = 0;
+    // round-synchronous: the lanes start their pieces together, so the piece set-up (divisions,
+    // per-axis ranges, first flux lookup) runs converged
+    for (int q0 = 0; q0 < total; q0 += 32) {
+      const int q = q0 + lane;
+      if (q < total) {
+        // owner hitter: first l with pre[l] > q
+        int l = 0;
 #pragma unroll
-      for (int s = 16; s > 0; s >>= 1)
-        if (pre[l + s - 1] <= q) l += s;
-      const int pi = q - (l ? pre[l - 1] : 0);
-      const Hitter& h = p.hit[h0 + l];
-      const double v0 = h.v0, v1 = h.v1, v2 = h.v2;
-      double lo_k = h.kin, hi_k = h.kout;
-      if (h.P > 1) {
-        const double vA = h.A == 0 ? v0 : (h.A == 1 ? v1 : v2);
-        const double rA = ddiv(1.0, vA);
-        if (pi > 0) lo_k = plane_k(p.g, h.A, h.jA + pi * h.stepG, rA);
-        if (pi < h.P - 1) hi_k = plane_k(p.g, h.A, h.jA + (pi + 1) * h.stepG, rA);
+        for (int s = 16; s > 0; s >>= 1)
+          if (pre[l + s - 1] <= q) l += s;
+        const int pi = q - (l ? pre[l - 1] : 0);
+        const Hitter& h = p.hit[h0 + l];
+        const double v0 = h.v0, v1 = h.v1, v2 = h.v2;
+        double lo_k = h.kin, hi_k = h.kout;
+        if (h.P > 1) {
+          const double vA = h.A == 0 ? v0 : (h.A == 1 ? v1 : v2);
+          const double rA = ddiv(1.0, vA);
+          if (pi > 0) lo_k = plane_k(p.g, h.A, h.jA + pi * h.stepG, rA);
+          if (pi < h.P - 1) hi_k = plane_k(p.g, h.A, h.jA + (pi + 1) * h.stepG, rA);
+        }
+        int nc;
+        const int ns = traj_walk<k3D>(p.g, fx, v0, v1, v2, lo_k, hi_k, h.oc, emit, &nc);
+        if (kStats) c_seg += ns;
       }
-      int nc;
-      const int ns = traj_walk(p.g, fx, v0, v1, v2, lo_k, hi_k, h.oc, emit, &nc);
-      if (kStats) c_seg += ns;
+      __syncwarp();
     }
-    __syncwarp();
   }
   if (kStats) flush_counter(p.stats + 3, c_seg);
 }
 
 // ---------------------------------------------------------------- B1-B3: one thread per event
+// fp32 fast path with a proven error bound: per (op, axis) the grid coordinate
+// t = x s - lo s is evaluated in fp32; |t32 - t64| < delta = c |q|max + d.  A pair whose t32 is
+// further than delta from every decision point (0, n and the integer bin edges) has exactly
+// the bin the fp64 definition gives; the rest (a ~1e-4 fraction) take the exact fp64 path.
+// Axes are tested in the order p.ord (fewest bins first: the thin L axis of a 2-D slice rejects
+// almost every pair after one row product).
+struct BinAxis32 {
+  float r0, r1, r2, s, los, c, d, n;
+};
+
 template <bool kPacked, bool kStats>
 __global__ void __launch_bounds__(kThreads)
 binmd_kernel(const __grid_constant__ BinParams p, const __grid_constant__ MatBlock mb) {
   __shared__ double sN[kMaxMats * 9];
+  __shared__ BinAxis32 sA[kMaxMats * 3];
   stage_binmd_mats(mb, sN);
+  __syncthreads();
+  for (int i = threadIdx.x; i < 3 * mb.nmat; i += blockDim.x) {
+    const int m = i / 3, a = p.ord[i - 3 * m];
+    const double* row = sN + 9 * m + 3 * a;
+    const double s = p.g.s[a], lo = p.g.lo[a];
+    const double sum = fabs(row[0]) + fabs(row[1]) + fabs(row[2]);
+    BinAxis32 ax;
+    ax.r0 = (float)row[0];
+    ax.r1 = (float)row[1];
+    ax.r2 = (float)row[2];
+    ax.s = (float)s;
+    ax.los = (float)(lo * s);
+    ax.c = (float)(1e-6 * s * sum);
+    ax.d = (float)(1e-6 * s * fabs(lo) + 1e-6 * (p.g.n[a] + 1.0));
+    ax.n = (float)p.g.n[a];
+    sA[i] = ax;
+  }
   __syncthreads();
   unsigned long long c_pairs = 0, c_in = 0;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
@@ -226,14 +319,40 @@ binmd_kernel(const __grid_constant__ BinParams p, const __grid_constant__ MatBlo
       q1 = __ldcs(ev + p.col_q + 1);
       q2 = __ldcs(ev + p.col_q + 2);
     }
-    const double wd = (double)w, d0 = (double)q0, d1 = (double)q1, d2 = (double)q2;
+    const float qm = fmaxf(fabsf(q0), fmaxf(fabsf(q1), fabsf(q2)));
     if (kStats) c_pairs += mb.nmat;
     for (int m = 0; m < mb.nmat; ++m) {
-      const int64_t b = event_bin(p.g, sN + 9 * m, d0, d1, d2);
-      if (b >= 0) {
-        atomicAdd(p.binmd + b, wd);
-        if (kStats) c_in += 1;
+      bool out = false, near = false;
+      int i0 = 0, i1 = 0, i2 = 0;
+#pragma unroll
+      for (int k = 0; k < 3; ++k) {
+        const BinAxis32 ax = sA[3 * m + k];
+        const float x = fmaf(ax.r2, q2, fmaf(ax.r1, q1, ax.r0 * q0));
+        const float t = fmaf(x, ax.s, -ax.los);
+        const float dl = fmaf(ax.c, qm, ax.d);
+        if (t < -dl || t >= ax.n + dl) {
+          out = true;
+          break;
+        }
+        const float fl = floorf(t);
+        const float fr = t - fl;
+        near = near || t < dl || t > ax.n - dl || fr < dl || fr > 1.0f - dl;
+        const int a = p.ord[k];
+        i0 = a == 0 ? (int)fl : i0;
+        i1 = a == 1 ? (int)fl : i1;
+        i2 = a == 2 ? (int)fl : i2;
       }
+      if (out) continue;
+      int b;
+      if (!near) {
+        b = i0 + p.g.n[0] * (i1 + p.g.n[1] * i2);
+      } else {  // within the error bound of a decision point: the fp64 definition decides
+        const int64_t be = event_bin(p.g, sN + 9 * m, (double)q0, (double)q1, (double)q2);
+        if (be < 0) continue;
+        b = (int)be;
+      }
+      atomicAdd(p.binmd + b, (double)w);
+      if (kStats) c_in += 1;
     }
   }
   if (kStats) {
@@ -288,7 +407,7 @@ struct RecordEmit {
   double* vals;
   int64_t max;
   int64_t n;
-  __device__ __forceinline__ void operator()(int64_t b, double val) {
+  __device__ __forceinline__ void operator()(int b, double val) {
     if (n < max) {
       bins[n] = b;
       vals[n] = val;
@@ -322,7 +441,7 @@ debug_traj_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ M
   }
   RecordEmit rec{seg_bins + t * max_segs, seg_vals + t * max_segs, max_segs, 0};
   int nc;
-  n_seg[t] = traj_walk(p.g, p.flux, v[0], v[1], v[2], kin, kout, dmul(px.w, sC[m]), rec, &nc);
+  n_seg[t] = traj_walk<true>(p.g, p.flux, v[0], v[1], v[2], kin, kout, dmul(px.w, sC[m]), rec, &nc);
   n_cross[t] = nc + 2;  // |L| = clip endpoints + crossings
 }
 
@@ -360,11 +479,11 @@ int grid_for(int64_t work, int num_sms, int per_sm, int threads = kThreads) {
   return (int)std::max<int64_t>(blocks, 1);
 }
 
-template <bool kSmemFlux, bool kStats>
+template <bool kSmemFlux, bool kStats, bool k3D>
 cudaError_t launch_walk(const MdnParams& p, int num_sms, cudaStream_t s) {
   const size_t smem = (kSmemFlux ? sizeof(double2) * p.flux.n + sizeof(int) * p.flux.ntab : 0) +
                       sizeof(int) * 32 * (kWalkThreads / 32);
-  auto k = mdnorm_walk_kernel<kSmemFlux, kStats>;
+  auto k = mdnorm_walk_kernel<kSmemFlux, kStats, k3D>;
   cudaError_t err = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (err != cudaSuccess) return err;
   int per_sm = 0;
@@ -376,11 +495,12 @@ cudaError_t launch_walk(const MdnParams& p, int num_sms, cudaStream_t s) {
 
 template <bool kStats>
 cudaError_t launch_cull(const MdnParams& p, const MatBlock& mb, int num_sms, cudaStream_t s) {
-  const size_t smem = sizeof(double) * 10 * (size_t)mb.nmat;
+  const size_t smem = (sizeof(double) * 10 + sizeof(CullMat)) * (size_t)mb.nmat +
+                      sizeof(uint32_t) * 128 * (kThreads / 32);
   auto k = mdnorm_cull_kernel<kStats>;
   cudaError_t err = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (err != cudaSuccess) return err;
-  k<<<grid_for(p.tlen, num_sms, 16), kThreads, smem, s>>>(p, mb);
+  k<<<grid_for(p.plen, num_sms, 8), kThreads, smem, s>>>(p, mb);
   return cudaGetLastError();
 }
 
@@ -399,15 +519,19 @@ cudaError_t launch_flux_table(const double2* kf, int n, int* tab, int ntab, doub
 }
 
 cudaError_t launch_mdnorm(const MdnParams& p, const MatBlock& mb, int num_sms, cudaStream_t s) {
-  if (p.tlen == 0 || mb.nmat <= 0) return cudaSuccess;
+  if (p.plen == 0 || mb.nmat <= 0) return cudaSuccess;
   cudaError_t err = cudaMemsetAsync(p.ctr, 0, sizeof(DevCounters), s);
   if (err != cudaSuccess) return err;
   err = p.stats ? launch_cull<true>(p, mb, num_sms, s) : launch_cull<false>(p, mb, num_sms, s);
   if (err != cudaSuccess) return err;
-  const bool smem_flux = p.flux.n <= kFluxSmemMax;
-  if (smem_flux)
-    return p.stats ? launch_walk<true, true>(p, num_sms, s) : launch_walk<true, false>(p, num_sms, s);
-  return p.stats ? launch_walk<false, true>(p, num_sms, s) : launch_walk<false, false>(p, num_sms, s);
+  // 2-D slices (a single bin on the last axis, "lBins=1") merge two crossing streams
+  const bool smem_flux = p.flux.n <= kFluxSmemMax, d3 = p.g.n[2] > 1;
+  if (smem_flux) {
+    if (d3) return p.stats ? launch_walk<true, true, true>(p, num_sms, s) : launch_walk<true, false, true>(p, num_sms, s);
+    return p.stats ? launch_walk<true, true, false>(p, num_sms, s) : launch_walk<true, false, false>(p, num_sms, s);
+  }
+  if (d3) return p.stats ? launch_walk<false, true, true>(p, num_sms, s) : launch_walk<false, false, true>(p, num_sms, s);
+  return p.stats ? launch_walk<false, true, false>(p, num_sms, s) : launch_walk<false, false, false>(p, num_sms, s);
 }
 
 cudaError_t launch_binmd(const BinParams& p, const MatBlock& mb, int num_sms, cudaStream_t s) {

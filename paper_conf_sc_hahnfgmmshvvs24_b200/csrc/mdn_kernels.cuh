@@ -60,7 +60,7 @@ struct MdnParams {
   // cull -> walk hand-off (production path)
   Hitter* hit;             // capacity >= slab length
   DevCounters* ctr;
-  uint32_t t0, tlen;       // slab of trajectory indices t = m * nshard + i
+  uint32_t p0, plen;       // slab: shard pixels [p0, p0 + plen), all matrices of the launch
 };
 
 struct BinParams {
@@ -68,6 +68,7 @@ struct BinParams {
   const float* events;
   int64_t nevents, stride;
   int32_t col_w, col_q;
+  int32_t ord[3];          // axis test order of the fp32 fast path (fewest bins first)
   int32_t acc_f32;
   double* binmd;           // fp64 histogram (nbins)
   unsigned long long* stats;  // nullptr, or [.., .., .., .., pairs, inside] (+= per launch)
@@ -78,7 +79,7 @@ cudaError_t launch_pixels_prepare(const double* dir, const double* solid, double
                                   cudaStream_t s);
 cudaError_t launch_flux_table(const double2* kf, int n, int* tab, int ntab, double k0, double cell,
                               cudaStream_t s);
-// MDNorm for trajectories [p.t0, p.t0 + p.tlen): cull (M1-M3) + piece walk (M3-M7).
+// MDNorm for shard pixels [p.p0, p.p0 + p.plen) x all matrices: cull (M1-M3) + piece walk (M3-M7).
 cudaError_t launch_mdnorm(const MdnParams& p, const MatBlock& mb, int num_sms, cudaStream_t s);
 cudaError_t launch_binmd(const BinParams& p, const MatBlock& mb, int num_sms, cudaStream_t s);
 cudaError_t launch_cross_section(const double* norm, const double* binmd, double* xs, int64_t nbins,
