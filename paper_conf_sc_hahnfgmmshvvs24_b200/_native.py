@@ -10,7 +10,8 @@ import os
 import re
 
 PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(PKG, "libmdnorm.so")
+# MDN_LIB_PATH: developer override to load an experimental build (tools/variants.sh)
+LIB_PATH = os.environ.get("MDN_LIB_PATH") or os.path.join(PKG, "libmdnorm.so")
 HEADER = os.path.join(os.path.dirname(PKG), "include", "mdnorm.h")
 
 MDN_OK, MDN_EINVAL, MDN_ENOMEM, MDN_ECUDA, MDN_ESTATE = 0, 1, 2, 3, 4

@@ -31,6 +31,7 @@ struct mdn_grid {
   int32_t nflux = 0, nftab = 0;
   double ftab_k0 = 0.0, ftab_inv_cell = 0.0;
   int ftab_nsteps = 0;
+  double flux_F_first = 0.0, flux_k_last = 0.0, flux_F_last = 0.0;
   mdn::Hitter* d_hit = nullptr;       // cull -> walk hand-off buffer
   uint32_t hit_cap = 0;
   mdn::DevCounters* d_ctr = nullptr;
@@ -172,7 +173,10 @@ mdn::MdnParams mdn_params(mdn_grid* g, double k_min, double k_max, int64_t pix_b
   p.nshard = nshard;
   p.flux.kf = g->d_flux;
   p.flux.tab = g->d_ftab;
-  p.flux.k0 = g->ftab_k0;
+  p.flux.k_first = g->ftab_k0;
+  p.flux.F_first = g->flux_F_first;
+  p.flux.k_last = g->flux_k_last;
+  p.flux.F_last = g->flux_F_last;
   p.flux.inv_cell = g->ftab_inv_cell;
   p.flux.n = g->nflux;
   p.flux.ntab = g->nftab;
@@ -340,6 +344,7 @@ mdn_status mdnorm_create_grid(int device, const double lo[3], const double hi[3]
     g->g.n[a] = (int32_t)nbins[a];
     g->g.w[a] = (hi[a] - lo[a]) / (double)nbins[a];  // IEEE double, same as the device would
     g->g.s[a] = 1.0 / g->g.w[a];
+    g->g.nd[a] = (double)nbins[a];
   }
   g->g.nbins = total;
   std::memcpy(g->W, W, sizeof g->W);
@@ -461,6 +466,9 @@ mdn_status mdnorm_set_flux(mdn_grid* g, int64_t n, const double* k, const double
   g->ftab_k0 = hk[0];
   g->ftab_inv_cell = 1.0 / cell;
   g->ftab_nsteps = nsteps;
+  g->flux_F_first = hF[0];
+  g->flux_k_last = hk[n - 1];
+  g->flux_F_last = hF[n - 1];
   return ok();
 }
 
@@ -478,7 +486,7 @@ mdn_status mdnorm_accumulate_runs(mdn_grid* g, const double UB[9], int32_t nruns
     if ((st = check_matrix(R + 9 * r, "R")) != MDN_OK) return st;
     if (!(std::isfinite(charge[r]) && charge[r] >= 0.0)) return fail(MDN_EINVAL, "charge[%d] = %g is not >= 0", r, charge[r]);
   }
-  int64_t nshard;
+  int64_t nshard = 0;
   if ((st = shard(g, pix_begin, pix_end, pix_stride, &nshard)) != MDN_OK) return st;
   DeviceGuard dg(g->device);
   cudaStream_t s = (cudaStream_t)stream;
@@ -589,7 +597,7 @@ mdn_status mdnorm_accumulate_matrices(mdn_grid* g, int32_t nmat, const double* M
   for (int m = 0; m < nmat; ++m)
     if (charge[m] < 0) return fail(MDN_EINVAL, "charge[%d] < 0", m);
   if ((st = check_krange(k_min, k_max)) != MDN_OK) return st;
-  int64_t nshard;
+  int64_t nshard = 0;
   if ((st = shard(g, pix_begin, pix_end, pix_stride, &nshard)) != MDN_OK) return st;
   DeviceGuard dg(g->device);
   MatBlock mb{};

@@ -19,6 +19,7 @@ namespace mdn {
 // SSE2: the same bits the device would produce).  Edge e_{a,j} = lo_a + j * w_a.
 struct GridC {
   double lo[3], hi[3], w[3], s[3];
+  double nd[3];  // n_a as double (the "t < n_a" tests)
   int32_t n[3];
   int32_t pad;
   int64_t nbins;
@@ -102,35 +103,33 @@ __device__ __forceinline__ bool compose_binmd(const double* UB, const double* S,
 struct FluxView {
   const double2* kf;  // (kappa_i, Phi_i)
   const int* tab;     // ntab cell start indices
-  double k0, inv_cell;
+  double k_first, F_first, k_last, F_last, inv_cell;
   int n, ntab, nsteps, pad;
 };
 
 __device__ __forceinline__ double flux_at(const FluxView& f, double x) {
-  const double2 first = f.kf[0], last = f.kf[f.n - 1];
-  if (x <= first.x) return first.y;
-  if (x >= last.x) return last.y;
-  const double u = (x - first.x) * f.inv_cell;  // any rounding: only selects the window
-  const int c = u < (double)(f.ntab - 1) ? (int)u : f.ntab - 1;
+  const double u = (x - f.k_first) * f.inv_cell;  // any rounding: only selects the window
+  const int c = u < 0.0 ? 0 : (u < (double)(f.ntab - 1) ? (int)u : f.ntab - 1);
   int lo = f.tab[max(c - 1, 0)];
   int hi = c + 2 < f.ntab ? f.tab[c + 2] + 1 : f.n - 1;
+  // invariant kappa_lo <= x < kappa_hi; extra steps on a closed window are no-ops, so the first
+  // four run unconditionally (no branches) and only very uneven tables need the loop
 #pragma unroll
-  for (int s = 0; s < 4; ++s) {  // invariant kappa_lo <= x < kappa_hi (nsteps is warp-uniform)
-    if (s < f.nsteps) {
-      const int mid = (lo + hi) >> 1;
-      const bool le = f.kf[mid].x <= x;
-      lo = le ? mid : lo;
-      hi = le ? hi : mid;
-    }
+  for (int s = 0; s < 4; ++s) {
+    const int mid = (lo + hi) >> 1;
+    const bool le = f.kf[mid].x <= x;
+    lo = le ? mid : lo;
+    hi = le ? hi : mid;
   }
-  for (int s = 4; s < f.nsteps; ++s) {  // only for very uneven knot spacing
+  for (int s = 4; s < f.nsteps; ++s) {
     const int mid = (lo + hi) >> 1;
     const bool le = f.kf[mid].x <= x;
     lo = le ? mid : lo;
     hi = le ? hi : mid;
   }
   const double2 a = f.kf[lo], b = f.kf[lo + 1];
-  return dadd(a.y, dmul(dsub(b.y, a.y), ddiv(dsub(x, a.x), dsub(b.x, a.x))));
+  const double F = dadd(a.y, dmul(dsub(b.y, a.y), ddiv(dsub(x, a.x), dsub(b.x, a.x))));
+  return x <= f.k_first ? f.F_first : (x >= f.k_last ? f.F_last : F);
 }
 
 // ------------------------------------------------------------------------------ M1-M2
@@ -295,8 +294,7 @@ __device__ __forceinline__ int traj_walk(const GridC& g, const FluxView& fx, dou
       const double t0 = dmul(dsub(dmul(km, v0), g.lo[0]), g.s[0]);
       const double t1 = dmul(dsub(dmul(km, v1), g.lo[1]), g.s[1]);
       const double t2 = dmul(dsub(dmul(km, v2), g.lo[2]), g.s[2]);
-      if (0.0 <= t0 && t0 < (double)g.n[0] && 0.0 <= t1 && t1 < (double)g.n[1] && 0.0 <= t2 &&
-          t2 < (double)g.n[2]) {
+      if (0.0 <= t0 && t0 < g.nd[0] && 0.0 <= t1 && t1 < g.nd[1] && 0.0 <= t2 && t2 < g.nd[2]) {
         const int b = __double2int_rz(t0) + g.n[0] * (__double2int_rz(t1) + g.n[1] * __double2int_rz(t2));
         emit(b, dmul(dsub(F2, F1), omega_c));
         ++nseg;
@@ -318,7 +316,7 @@ __device__ __forceinline__ int64_t event_bin(const GridC& g, const double* N, do
   for (int a = 0; a < 3; ++a) {
     double x = row_dot(N + 3 * a, q0, q1, q2);
     double t = dmul(dsub(x, g.lo[a]), g.s[a]);
-    if (!(0.0 <= t && t < (double)g.n[a])) return -1;
+    if (!(0.0 <= t && t < g.nd[a])) return -1;
     idx[a] = __double2int_rz(t);
   }
   return (int64_t)idx[0] + (int64_t)g.n[0] * ((int64_t)idx[1] + (int64_t)g.n[1] * idx[2]);

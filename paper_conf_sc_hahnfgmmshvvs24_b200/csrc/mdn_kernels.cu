@@ -20,8 +20,14 @@ namespace mdn {
 
 namespace {
 
+#ifndef MDN_WALK_THREADS
+#define MDN_WALK_THREADS 512
+#endif
+#ifndef MDN_WALK_MINB
+#define MDN_WALK_MINB 2
+#endif
 constexpr int kThreads = 256;
-constexpr int kWalkThreads = 512;
+constexpr int kWalkThreads = MDN_WALK_THREADS;
 constexpr unsigned kFull = 0xffffffffu;
 
 __device__ __forceinline__ void stage_mdnorm_mats(const MatBlock& mb, double* sM, double* sC) {
@@ -66,9 +72,10 @@ struct AtomicEmit {
 // read once; matrices are warp-uniform smem broadcasts).  A conservative fp32 slab test with a
 // proven error margin rejects most misses without any fp64 division; every
 // survivor gets the exact fp64 v and clip, so the hit decision is the definition's.
-struct CullMat {
+struct alignas(16) CullMat {
   float M[9];
-  float delta[3];  // per-axis margin of the fp32 test
+  float lot[3], hit[3];  // per-axis fp32 acceptance window [lo - delta, hi + delta)
+  float pad;
 };
 
 template <bool kStats>
@@ -88,13 +95,13 @@ mdnorm_cull_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ 
         sum += fabs(sM[9 * m + 3 * a + i]);
       }
       // |q_i| <= 2; fp32 v and x = k v are within 1e-6 kmax sum|M_a| of the exact values
-      sF[m].delta[a] = (float)(4e-6 * p.kmax * sum + 1e-6 * (fabs(p.g.lo[a]) + fabs(p.g.hi[a])) + 1e-30);
+      const double delta = 4e-6 * p.kmax * sum + 1e-6 * (fabs(p.g.lo[a]) + fabs(p.g.hi[a])) + 1e-30;
+      sF[m].lot[a] = (float)p.g.lo[a] - (float)delta;
+      sF[m].hit[a] = (float)p.g.hi[a] + (float)delta;
     }
   }
   __syncthreads();
   const float kmin32 = (float)p.kmin, kmax32 = (float)p.kmax;
-  const float lo32[3] = {(float)p.g.lo[0], (float)p.g.lo[1], (float)p.g.lo[2]};
-  const float hi32[3] = {(float)p.g.hi[0], (float)p.g.hi[1], (float)p.g.hi[2]};
   const int lane = threadIdx.x & 31;
   // per-warp ring of fp32 survivors (pixel offset, matrix); the exact fp64 path runs only when
   // 32 of them are queued, so it executes with the whole warp converged
@@ -133,8 +140,8 @@ mdnorm_cull_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ 
           const int A = a2 ? 2 : (a1 ? 1 : 0);
           int P = 1, G = 1;
           if (total + 1 > kPieceSegs && sa.cnt > 1) {
-            const int want = (total + kPieceSegs) / kPieceSegs;  // ceil((total + 1) / target)
-            G = max(1, (sa.cnt + want - 1) / want);
+            // G crossings of A per piece bring ~G (total + 1) / cA segments: aim at kPieceSegs
+            G = max(1, (kPieceSegs * sa.cnt + (total + 1) / 2) / (total + 1));
             P = (sa.cnt + G - 1) / G;
           }
           h.v0 = v0; h.v1 = v1; h.v2 = v2; h.kin = kin; h.kout = kout;
@@ -170,14 +177,14 @@ mdnorm_cull_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ 
     const bool live = valid && px.w != 0.0;  // masked pixels contribute 0 (reading #16)
     const float q0 = (float)px.x, q1 = (float)px.y, q2 = (float)px.z;
     for (int m = 0; m < mb.nmat; ++m) {
-      const CullMat& cm = sF[m];
+      const CullMat cm = sF[m];
       bool maybe = live;
 #pragma unroll
-      for (int a = 0; a < 3; ++a) {
+      for (int a = 0; a < 3; ++a) {  // branch-free: all three slabs
         const float v = fmaf(cm.M[3 * a + 2], q2, fmaf(cm.M[3 * a + 1], q1, cm.M[3 * a] * q0));
         const float xa = kmin32 * v, xb = kmax32 * v;
         const float xl = fminf(xa, xb), xh = fmaxf(xa, xb);
-        maybe = maybe && !(xh < lo32[a] - cm.delta[a] || xl >= hi32[a] + cm.delta[a]);
+        maybe &= (xh >= cm.lot[a]) & (xl < cm.hit[a]);
       }
       const unsigned mask = __ballot_sync(kFull, maybe);
       if (maybe) {
@@ -199,7 +206,7 @@ mdnorm_cull_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ 
 
 // ---------------------------------------------------------------- M3-M7: balanced piece walk
 template <bool kSmemFlux, bool kStats, bool k3D>
-__global__ void __launch_bounds__(kWalkThreads, 2)
+__global__ void __launch_bounds__(kWalkThreads, MDN_WALK_MINB)
 mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
   extern __shared__ double2 wsm[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -305,56 +312,144 @@ binmd_kernel(const __grid_constant__ BinParams p, const __grid_constant__ MatBlo
     sA[i] = ax;
   }
   __syncthreads();
-  unsigned long long c_pairs = 0, c_in = 0;
-  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < p.nevents; e += stride) {
-    float w, q0, q1, q2;
-    if (kPacked) {
-      const float4 ev = __ldcs(reinterpret_cast<const float4*>(p.events) + e);
-      w = ev.x; q0 = ev.y; q1 = ev.z; q2 = ev.w;
-    } else {
-      const float* ev = p.events + e * p.stride;
-      w = __ldcs(ev + p.col_w);
-      q0 = __ldcs(ev + p.col_q);
-      q1 = __ldcs(ev + p.col_q + 1);
-      q2 = __ldcs(ev + p.col_q + 2);
-    }
-    const float qm = fmaxf(fabsf(q0), fmaxf(fabsf(q1), fabsf(q2)));
-    if (kStats) c_pairs += mb.nmat;
-    for (int m = 0; m < mb.nmat; ++m) {
-      bool out = false, near = false;
-      int i0 = 0, i1 = 0, i2 = 0;
-#pragma unroll
-      for (int k = 0; k < 3; ++k) {
-        const BinAxis32 ax = sA[3 * m + k];
-        const float x = fmaf(ax.r2, q2, fmaf(ax.r1, q1, ax.r0 * q0));
-        const float t = fmaf(x, ax.s, -ax.los);
-        const float dl = fmaf(ax.c, qm, ax.d);
-        if (t < -dl || t >= ax.n + dl) {
-          out = true;
-          break;
-        }
-        const float fl = floorf(t);
-        const float fr = t - fl;
-        near = near || t < dl || t > ax.n - dl || fr < dl || fr > 1.0f - dl;
-        const int a = p.ord[k];
-        i0 = a == 0 ? (int)fl : i0;
-        i1 = a == 1 ? (int)fl : i1;
-        i2 = a == 2 ? (int)fl : i2;
+  // Ops whose first-tested row is the same fp32 vector give the same t on that axis, so the
+  // test is done once per class (symmetry ops map L -> +-L: 2 classes for 6/mmm on a slice).
+  __shared__ int sRep[kMaxMats], sCid[kMaxMats], sCls[kMaxMats + 1], sMem[kMaxMats];
+  __shared__ int sNcls;
+  for (int m = threadIdx.x; m < mb.nmat; m += blockDim.x) {
+    const BinAxis32 am = sA[3 * m];
+    int rep = m;
+    for (int r = 0; r < m; ++r) {
+      const BinAxis32 ar = sA[3 * r];
+      if (ar.r0 == am.r0 && ar.r1 == am.r1 && ar.r2 == am.r2 &&
+          __float_as_uint(ar.r0) == __float_as_uint(am.r0) && __float_as_uint(ar.r1) == __float_as_uint(am.r1) &&
+          __float_as_uint(ar.r2) == __float_as_uint(am.r2)) {
+        rep = r;
+        break;
       }
-      if (out) continue;
-      int b;
-      if (!near) {
-        b = i0 + p.g.n[0] * (i1 + p.g.n[1] * i2);
-      } else {  // within the error bound of a decision point: the fp64 definition decides
-        const int64_t be = event_bin(p.g, sN + 9 * m, (double)q0, (double)q1, (double)q2);
-        if (be < 0) continue;
-        b = (int)be;
-      }
-      atomicAdd(p.binmd + b, (double)w);
-      if (kStats) c_in += 1;
     }
+    sRep[m] = rep;
   }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    int ncls = 0;
+    for (int m = 0; m < mb.nmat; ++m) {
+      sCid[m] = sRep[m] == m ? ncls++ : sCid[sRep[m]];
+    }
+    for (int c = 0; c <= ncls; ++c) sCls[c] = 0;
+    for (int m = 0; m < mb.nmat; ++m) sCls[sCid[m] + 1] += 1;
+    for (int c = 0; c < ncls; ++c) sCls[c + 1] += sCls[c];
+    int fill[kMaxMats];
+    for (int c = 0; c < ncls; ++c) fill[c] = sCls[c];
+    for (int m = 0; m < mb.nmat; ++m) sMem[fill[sCid[m]]++] = m;
+    sNcls = ncls;
+  }
+  __syncthreads();
+  const int ncls = sNcls;
+  const int a0 = p.ord[0], a1 = p.ord[1], a2 = p.ord[2];
+  const int lane = threadIdx.x & 31;
+  // per-warp queue of (event, class) pairs that pass the class test: their member loop runs
+  // only when 32 are queued, with the warp converged
+  __shared__ float4 sQv[(kThreads / 32) * 64];
+  __shared__ int sQc[(kThreads / 32) * 64];
+  float4* qv = sQv + (threadIdx.x >> 5) * 64;
+  int* qc = sQc + (threadIdx.x >> 5) * 64;
+  int qhead = 0, qcnt = 0;
+  unsigned long long c_pairs = 0, c_in = 0;
+
+  auto drain = [&](int n) {
+    __syncwarp();
+    if (lane < n) {
+      const int slot = (qhead + lane) & 63;
+      const float4 ev = qv[slot];
+      const int c = qc[slot];
+      const float w = ev.x, q0 = ev.y, q1 = ev.z, q2 = ev.w;
+      const float qm = fmaxf(fabsf(q0), fmaxf(fabsf(q1), fabsf(q2)));
+      const int j0 = sCls[c], j1 = sCls[c + 1];
+      const BinAxis32 ax = sA[3 * sMem[j0]];
+      const float x = fmaf(ax.r2, q2, fmaf(ax.r1, q1, ax.r0 * q0));
+      const float t = fmaf(x, ax.s, -ax.los);
+      const float dl = fmaf(ax.c, qm, ax.d);
+      const float fl = floorf(t);
+      const float fr = t - fl;
+      const bool near0 = t < dl || t > ax.n - dl || fr < dl || fr > 1.0f - dl;
+      const int ifirst = (int)fl;
+      for (int j = j0; j < j1; ++j) {
+        const int m = sMem[j];
+        bool out = false, near = near0;
+        int ik[3] = {ifirst, 0, 0};
+#pragma unroll
+        for (int k = 1; k < 3; ++k) {
+          const BinAxis32 bx = sA[3 * m + k];
+          const float xk = fmaf(bx.r2, q2, fmaf(bx.r1, q1, bx.r0 * q0));
+          const float tk = fmaf(xk, bx.s, -bx.los);
+          const float dk = fmaf(bx.c, qm, bx.d);
+          out = out || tk < -dk || tk >= bx.n + dk;
+          const float fk = floorf(tk);
+          const float rk = tk - fk;
+          near = near || tk < dk || tk > bx.n - dk || rk < dk || rk > 1.0f - dk;
+          ik[k] = (int)fk;
+        }
+        if (out) continue;
+        // bin indices back in axis order (ord is a permutation of 0, 1, 2)
+        const int i0 = a0 == 0 ? ik[0] : (a1 == 0 ? ik[1] : ik[2]);
+        const int i1 = a0 == 1 ? ik[0] : (a1 == 1 ? ik[1] : ik[2]);
+        const int i2 = a0 == 2 ? ik[0] : (a1 == 2 ? ik[1] : ik[2]);
+        (void)a2;
+        int b;
+        if (!near) {
+          b = i0 + p.g.n[0] * (i1 + p.g.n[1] * i2);
+        } else {  // within the error bound of a decision point: the fp64 definition decides
+          const int64_t be = event_bin(p.g, sN + 9 * m, (double)q0, (double)q1, (double)q2);
+          if (be < 0) continue;
+          b = (int)be;
+        }
+        atomicAdd(p.binmd + b, (double)w);
+        if (kStats) c_in += 1;
+      }
+    }
+    qhead = (qhead + n) & 63;
+    qcnt -= n;
+    __syncwarp();
+  };
+
+  auto load = [&](int64_t e) {
+    if (kPacked) return __ldcs(reinterpret_cast<const float4*>(p.events) + e);
+    const float* ev = p.events + e * p.stride;
+    return make_float4(__ldcs(ev + p.col_w), __ldcs(ev + p.col_q), __ldcs(ev + p.col_q + 1),
+                       __ldcs(ev + p.col_q + 2));
+  };
+
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  int64_t base = (int64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31);  // warp-uniform
+  float4 cur = make_float4(0.f, 0.f, 0.f, 0.f);
+  if (base + lane < p.nevents) cur = load(base + lane);
+  for (; base < p.nevents; base += stride) {
+    const bool valid = base + lane < p.nevents;
+    float4 nxt = make_float4(0.f, 0.f, 0.f, 0.f);  // software prefetch of the next event
+    if (base + stride + lane < p.nevents) nxt = load(base + stride + lane);
+    const float q0 = cur.y, q1 = cur.z, q2 = cur.w;
+    const float qm = fmaxf(fabsf(q0), fmaxf(fabsf(q1), fabsf(q2)));
+    if (kStats && valid) c_pairs += mb.nmat;
+    for (int c = 0; c < ncls; ++c) {
+      // first-tested axis, once for the whole class
+      const BinAxis32 ax = sA[3 * sMem[sCls[c]]];
+      const float x = fmaf(ax.r2, q2, fmaf(ax.r1, q1, ax.r0 * q0));
+      const float t = fmaf(x, ax.s, -ax.los);
+      const float dl = fmaf(ax.c, qm, ax.d);
+      const bool pass = valid && t >= -dl && t < ax.n + dl;
+      const unsigned mask = __ballot_sync(kFull, pass);
+      if (pass) {
+        const int slot = (qhead + qcnt + __popc(mask & ((1u << lane) - 1u))) & 63;
+        qv[slot] = cur;
+        qc[slot] = c;
+      }
+      qcnt += __popc(mask);
+      if (qcnt >= 32) drain(32);
+    }
+    cur = nxt;
+  }
+  if (qcnt > 0) drain(qcnt);
   if (kStats) {
     flush_counter(p.stats + 4, c_pairs);
     flush_counter(p.stats + 5, c_in);

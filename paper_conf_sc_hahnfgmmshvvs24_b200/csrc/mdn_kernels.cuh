@@ -11,7 +11,10 @@ constexpr int kMaxOps = 48;           // MDN_MAX_OPS
 constexpr int kMaxMats = 64;          // MDN_MAX_MATS
 constexpr int kRunsPerLaunch = 16;    // runs composed per MDNorm launch (batched API)
 constexpr int kFluxSmemMax = 4096;    // flux knots staged in shared memory (64 KB of double2)
-constexpr int kPieceSegs = 24;        // target segments per work piece (load balance, M4-M7)
+#ifndef MDN_PIECE_SEGS
+#define MDN_PIECE_SEGS 24
+#endif
+constexpr int kPieceSegs = MDN_PIECE_SEGS;  // target segments per work piece (load balance, M4-M7)
 
 // Matrices for one launch, passed by value as a __grid_constant__ kernel parameter (sm_70+
 // kernels accept up to 32 KB of parameters; CUDA >= 12.1).  Either compose (UB, W, ops, R) on
