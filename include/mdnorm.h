@@ -44,8 +44,9 @@
  *  - Precision: geometry (matrices, clip, crossings, midpoints, bin indices, flux
  *    interpolation) is IEEE fp64 without FMA contraction, so crossing counts and bin indices are
  *    bit-identical to the fp64 oracle.  Global histograms are fp64.  mdn_acc selects the
- *    precision of the per-CTA privatised partial sums (MDN_ACC_F64: fp64 end to end;
- *    MDN_ACC_F32: fp32 partials folded into the fp64 histogram, BASELINE north_star fp32 mode).
+ *    precision of privatised partial sums: MDN_ACC_F64 = fp64 end to end (this build);
+ *    MDN_ACC_F32 (fp32 partials folded into the fp64 histogram, BASELINE north_star fp32 mode)
+ *    is reserved and currently rejected with MDN_EINVAL.
  */
 #ifndef MDNORM_H
 #define MDNORM_H

@@ -288,6 +288,59 @@ struct BinAxis32 {
   float r0, r1, r2, s, los, c, d, n;
 };
 
+// Member loop of one queued (event, class) pair: the remaining two axes of every op of the
+// class, bin and fp64 red.add.  Out of line so that its constants are not hoisted into the
+// class-test loop.  Returns the number of (event, op) pairs that landed inside the grid.
+__device__ __noinline__ unsigned binmd_members(const BinParams& p, const double* sN, const BinAxis32* sA,
+                                               const int* sCls, const int* sMem, float4 ev, int c, int a0,
+                                               int a1) {
+  const float w = ev.x, q0 = ev.y, q1 = ev.z, q2 = ev.w;
+  const float qm = fmaxf(fabsf(q0), fmaxf(fabsf(q1), fabsf(q2)));
+  const int j0 = sCls[c], j1 = sCls[c + 1];
+  const BinAxis32 ax = sA[3 * sMem[j0]];
+  const float x = fmaf(ax.r2, q2, fmaf(ax.r1, q1, ax.r0 * q0));
+  const float t = fmaf(x, ax.s, -ax.los);
+  const float dl = fmaf(ax.c, qm, ax.d);
+  const float fl = floorf(t);
+  const float fr = t - fl;
+  const bool near0 = t < dl || t > ax.n - dl || fr < dl || fr > 1.0f - dl;
+  const int ifirst = (int)fl;
+  unsigned inside = 0;
+  for (int j = j0; j < j1; ++j) {
+    const int m = sMem[j];
+    bool out = false, near = near0;
+    int ik[3] = {ifirst, 0, 0};
+#pragma unroll
+    for (int k = 1; k < 3; ++k) {
+      const BinAxis32 bx = sA[3 * m + k];
+      const float xk = fmaf(bx.r2, q2, fmaf(bx.r1, q1, bx.r0 * q0));
+      const float tk = fmaf(xk, bx.s, -bx.los);
+      const float dk = fmaf(bx.c, qm, bx.d);
+      out = out || tk < -dk || tk >= bx.n + dk;
+      const float fk = floorf(tk);
+      const float rk = tk - fk;
+      near = near || tk < dk || tk > bx.n - dk || rk < dk || rk > 1.0f - dk;
+      ik[k] = (int)fk;
+    }
+    if (out) continue;
+    // bin indices back in axis order (ord is a permutation of 0, 1, 2)
+    const int i0 = a0 == 0 ? ik[0] : (a1 == 0 ? ik[1] : ik[2]);
+    const int i1 = a0 == 1 ? ik[0] : (a1 == 1 ? ik[1] : ik[2]);
+    const int i2 = a0 == 2 ? ik[0] : (a1 == 2 ? ik[1] : ik[2]);
+    int b;
+    if (!near) {
+      b = i0 + p.g.n[0] * (i1 + p.g.n[1] * i2);
+    } else {  // within the error bound of a decision point: the fp64 definition decides
+      const int64_t be = event_bin(p.g, sN + 9 * m, (double)q0, (double)q1, (double)q2);
+      if (be < 0) continue;
+      b = (int)be;
+    }
+    atomicAdd(p.binmd + b, (double)w);
+    ++inside;
+  }
+  return inside;
+}
+
 template <bool kPacked, bool kStats>
 __global__ void __launch_bounds__(kThreads)
 binmd_kernel(const __grid_constant__ BinParams p, const __grid_constant__ MatBlock mb) {
@@ -357,56 +410,12 @@ binmd_kernel(const __grid_constant__ BinParams p, const __grid_constant__ MatBlo
   int qhead = 0, qcnt = 0;
   unsigned long long c_pairs = 0, c_in = 0;
 
+  (void)a2;
   auto drain = [&](int n) {
     __syncwarp();
     if (lane < n) {
       const int slot = (qhead + lane) & 63;
-      const float4 ev = qv[slot];
-      const int c = qc[slot];
-      const float w = ev.x, q0 = ev.y, q1 = ev.z, q2 = ev.w;
-      const float qm = fmaxf(fabsf(q0), fmaxf(fabsf(q1), fabsf(q2)));
-      const int j0 = sCls[c], j1 = sCls[c + 1];
-      const BinAxis32 ax = sA[3 * sMem[j0]];
-      const float x = fmaf(ax.r2, q2, fmaf(ax.r1, q1, ax.r0 * q0));
-      const float t = fmaf(x, ax.s, -ax.los);
-      const float dl = fmaf(ax.c, qm, ax.d);
-      const float fl = floorf(t);
-      const float fr = t - fl;
-      const bool near0 = t < dl || t > ax.n - dl || fr < dl || fr > 1.0f - dl;
-      const int ifirst = (int)fl;
-      for (int j = j0; j < j1; ++j) {
-        const int m = sMem[j];
-        bool out = false, near = near0;
-        int ik[3] = {ifirst, 0, 0};
-#pragma unroll
-        for (int k = 1; k < 3; ++k) {
-          const BinAxis32 bx = sA[3 * m + k];
-          const float xk = fmaf(bx.r2, q2, fmaf(bx.r1, q1, bx.r0 * q0));
-          const float tk = fmaf(xk, bx.s, -bx.los);
-          const float dk = fmaf(bx.c, qm, bx.d);
-          out = out || tk < -dk || tk >= bx.n + dk;
-          const float fk = floorf(tk);
-          const float rk = tk - fk;
-          near = near || tk < dk || tk > bx.n - dk || rk < dk || rk > 1.0f - dk;
-          ik[k] = (int)fk;
-        }
-        if (out) continue;
-        // bin indices back in axis order (ord is a permutation of 0, 1, 2)
-        const int i0 = a0 == 0 ? ik[0] : (a1 == 0 ? ik[1] : ik[2]);
-        const int i1 = a0 == 1 ? ik[0] : (a1 == 1 ? ik[1] : ik[2]);
-        const int i2 = a0 == 2 ? ik[0] : (a1 == 2 ? ik[1] : ik[2]);
-        (void)a2;
-        int b;
-        if (!near) {
-          b = i0 + p.g.n[0] * (i1 + p.g.n[1] * i2);
-        } else {  // within the error bound of a decision point: the fp64 definition decides
-          const int64_t be = event_bin(p.g, sN + 9 * m, (double)q0, (double)q1, (double)q2);
-          if (be < 0) continue;
-          b = (int)be;
-        }
-        atomicAdd(p.binmd + b, (double)w);
-        if (kStats) c_in += 1;
-      }
+      c_in += binmd_members(p, sN, sA, sCls, sMem, qv[slot], qc[slot], a0, a1);
     }
     qhead = (qhead + n) & 63;
     qcnt -= n;

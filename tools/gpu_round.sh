@@ -1,5 +1,5 @@
 #!/bin/bash
-# One GPU session: smoke, GPU tests, bench, ncu launch list and a full capture of the top
+# One GPU session: smoke, GPU tests, bench, ncu launch list and a full capture of the hot
 # kernels.  Logs land in gpurun_out/.  Usage (from this container):
 #   gpurun --timeout 2400 -- 'bash tools/gpu_round.sh [quick]'
 set -u
@@ -14,7 +14,8 @@ if [ "$MODE" = "quick" ]; then exit 0; fi
 echo "== ncu launch list"
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches.csv \
   python bench.py --steps 2 --warmup 3 --no-cpu-baseline > $OUT/ncu_launch_bench.log 2>&1; echo "ncu list rc=$?"
-echo "== ncu full (mdnorm, binmd)"
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:'mdnorm_kernel|binmd_kernel' -s 4 -c 2 \
+echo "== ncu full (cull, walk, binmd, xs)"
+timeout 900 ncu --set full --clock-control none --import-source on \
+  -k regex:'mdnorm_cull_kernel|mdnorm_walk_kernel|binmd_kernel|xs_kernel' -s 8 -c 4 \
   -o $OUT/prof_full -f python bench.py --steps 2 --warmup 3 --no-cpu-baseline > $OUT/ncu_full.log 2>&1; echo "ncu full rc=$?"
 ls -la $OUT
