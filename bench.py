@@ -390,17 +390,25 @@ def main():
     ap.add_argument("--cpu-stride", type=int, default=2, help="oracle sample: every n-th pixel and event")
     ap.add_argument("--ref-stride", type=int, default=8, help="--impl reference per-step sample stride")
     ap.add_argument("--json-out", default=None)
+    ap.add_argument("--dist-backend", default="nccl",
+                    help="nccl (production); gloo + MDN_BENCH_SHARED_GPU=1 exercises the N>1 code "
+                         "path with every rank on GPU 0 (tests only; not a performance number)")
     args = ap.parse_args()
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if os.environ.get("MDN_BENCH_SHARED_GPU") == "1":
+        local_rank = 0
     if args.impl == "reference":
         return run_reference(args, rank, world)
     if world > 1:
         import torch
         import torch.distributed as dist
         torch.cuda.set_device(local_rank)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        if args.dist_backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        else:
+            dist.init_process_group(args.dist_backend)
     try:
         return run_ours(args, rank, world, local_rank)
     finally:

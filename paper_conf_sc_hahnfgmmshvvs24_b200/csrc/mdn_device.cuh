@@ -12,6 +12,10 @@
 #include <cuda_runtime.h>
 #include <math_constants.h>
 
+#ifndef MDN_MERGE2D_BRANCH
+#define MDN_MERGE2D_BRANCH 0  // 2-D slices: branchy two-stream merge instead of selects
+#endif
+
 namespace mdn {
 
 // ------------------------------------------------------------------------------ grid constants
@@ -108,26 +112,31 @@ struct FluxView {
 };
 
 __device__ __forceinline__ double flux_at(const FluxView& f, double x) {
-  const double u = (x - f.k_first) * f.inv_cell;  // any rounding: only selects the window
-  const int c = u < 0.0 ? 0 : (u < (double)(f.ntab - 1) ? (int)u : f.ntab - 1);
-  int lo = f.tab[max(c - 1, 0)];
-  int hi = c + 2 < f.ntab ? f.tab[c + 2] + 1 : f.n - 1;
-  // invariant kappa_lo <= x < kappa_hi; extra steps on a closed window are no-ops, so the first
-  // four run unconditionally (no branches) and only very uneven tables need the loop
+#ifdef MDN_EXP_NOFLUX  // timing experiment only (wrong results): F(x) = x
+  return x;
+#endif
+  // Cell of x from an approximate u (relative error ~1e-16, i.e. ~1e-12 cells): unless u is
+  // within 1e-9 of a cell boundary the cell c is exact and the window is [tab[c], tab[c+1] + 1]
+  // (the knots of one cell); near a boundary it is widened by one cell on each side.
+  const double u = fmin(fmax((x - f.k_first) * f.inv_cell, 0.0), (double)(f.ntab - 1));
+  const double cf = floor(u);
+  const int c = (int)cf;
+  const double fr = u - cf;
+  const bool edge = fr < 1e-9 || fr > 1.0 - 1e-9;
+  const int lo = f.tab[edge ? max(c - 1, 0) : c];
+  const int ch = edge ? c + 2 : c + 1;
+  const int hi = ch < f.ntab ? f.tab[ch] + 1 : f.n - 1;
+  // invariant kappa_lo <= x < kappa_hi; i = lo + #{t >= 1 : kappa_{lo+t} <= x}: three
+  // independent probes cover a cell of up to 3 knots, the loop finishes denser cells
+  int i = lo;
 #pragma unroll
-  for (int s = 0; s < 4; ++s) {
-    const int mid = (lo + hi) >> 1;
-    const bool le = f.kf[mid].x <= x;
-    lo = le ? mid : lo;
-    hi = le ? hi : mid;
+  for (int t = 1; t <= 3; ++t) {
+    const int j = lo + t;
+    if (j < hi) i += f.kf[j].x <= x ? 1 : 0;
   }
-  for (int s = 4; s < f.nsteps; ++s) {
-    const int mid = (lo + hi) >> 1;
-    const bool le = f.kf[mid].x <= x;
-    lo = le ? mid : lo;
-    hi = le ? hi : mid;
-  }
-  const double2 a = f.kf[lo], b = f.kf[lo + 1];
+  if (i == lo + 3)
+    while (i + 1 < hi && f.kf[i + 1].x <= x) ++i;
+  const double2 a = f.kf[i], b = f.kf[i + 1];
   const double F = dadd(a.y, dmul(dsub(b.y, a.y), ddiv(dsub(x, a.x), dsub(b.x, a.x))));
   return x <= f.k_first ? f.F_first : (x >= f.k_last ? f.F_last : F);
 }
@@ -266,30 +275,46 @@ __device__ __forceinline__ int traj_walk(const GridC& g, const FluxView& fx, dou
   *ncross = total;
   double k1 = lo_k, F1 = flux_at(fx, lo_k);
   int nseg = 0;
-  for (int left = total; left >= 0; --left) {
-    // smallest pending crossing (ties: lowest axis first; equal values give a skipped
-    // zero-length segment, so the order among ties never matters)
+  int left = total;
+  // next entry of L: the smallest pending crossing (ties: lowest axis first; equal values give
+  // a skipped zero-length segment, so the order among ties never matters), then hi_k
+  auto next = [&]() -> double {
+    if (left == 0) return hi_k;
+    --left;
+    if (!k3D) {  // 2-D slice: two streams
+      if (c0.nk <= c1.nk) {
+        const double k = c0.nk;
+        c0.jd += c0.stepd;
+        --c0.cnt;
+        c0.nk = c0.cnt > 0 ? dmul(dadd(g.lo[0], dmul(c0.jd, g.w[0])), c0.r) : CUDART_INF;
+        return k;
+      }
+      const double k = c1.nk;
+      c1.jd += c1.stepd;
+      --c1.cnt;
+      c1.nk = c1.cnt > 0 ? dmul(dadd(g.lo[1], dmul(c1.jd, g.w[1])), c1.r) : CUDART_INF;
+      return k;
+    }
+    // three streams, selects only: advance the chosen axis with one plane evaluation
     const bool s01 = c1.nk < c0.nk;
     const double m01 = s01 ? c1.nk : c0.nk;
-    const bool s2 = k3D && c2.nk < m01;
+    const bool s2 = c2.nk < m01;
     const bool p0 = !s2 && !s01, p1 = !s2 && s01;
-    double k2 = s2 ? c2.nk : m01;
-    // advance the chosen axis (selects, one plane evaluation)
+    const double k = s2 ? c2.nk : m01;
     const double jd = (p0 ? c0.jd + c0.stepd : (p1 ? c1.jd + c1.stepd : c2.jd + c2.stepd));
     const int cnt = (p0 ? c0.cnt : (p1 ? c1.cnt : c2.cnt)) - 1;
     const double lo = p0 ? g.lo[0] : (p1 ? g.lo[1] : g.lo[2]);
     const double w = p0 ? g.w[0] : (p1 ? g.w[1] : g.w[2]);
     const double r = p0 ? c0.r : (p1 ? c1.r : c2.r);
     const double nk = cnt > 0 ? dmul(dadd(lo, dmul(jd, w)), r) : CUDART_INF;
-    if (left > 0) {
-      if (p0) { c0.jd = jd; c0.cnt = cnt; c0.nk = nk; }
-      if (p1) { c1.jd = jd; c1.cnt = cnt; c1.nk = nk; }
-      if (k3D && s2) { c2.jd = jd; c2.cnt = cnt; c2.nk = nk; }
-    } else {
-      k2 = hi_k;
-    }
+    if (p0) { c0.jd = jd; c0.cnt = cnt; c0.nk = nk; }
+    if (p1) { c1.jd = jd; c1.cnt = cnt; c1.nk = nk; }
+    if (s2) { c2.jd = jd; c2.cnt = cnt; c2.nk = nk; }
+    return k;
+  };
+  // segment (k1, k2) if it has positive length: midpoint bin (M6) and value (M7)
+  auto segment = [&](double k2, double F2) {
     if (k2 > k1) {
-      const double F2 = flux_at(fx, k2);
       const double km = dmul(0.5, dadd(k1, k2));
       const double t0 = dmul(dsub(dmul(km, v0), g.lo[0]), g.s[0]);
       const double t1 = dmul(dsub(dmul(km, v1), g.lo[1]), g.s[1]);
@@ -302,6 +327,24 @@ __device__ __forceinline__ int traj_walk(const GridC& g, const FluxView& fx, dou
       k1 = k2;
       F1 = F2;
     }
+  };
+  // L has total + 1 entries after lo_k.  3-D: two at a time, so that their flux look-ups (the
+  // longest dependency chain) are independent and overlap; 2-D slices (two streams, fewer live
+  // registers) measured faster one at a time.
+  int rem = total + 1;
+  if (k3D) {
+    for (; rem >= 2; rem -= 2) {
+      const double ka = next();
+      const double kb = next();
+      const double Fa = flux_at(fx, ka);
+      const double Fb = flux_at(fx, kb);
+      segment(ka, Fa);
+      segment(kb, Fb);
+    }
+  }
+  for (; rem >= 1; --rem) {
+    const double ka = next();
+    segment(ka, flux_at(fx, ka));
   }
   return nseg;
 }

@@ -21,13 +21,16 @@ namespace mdn {
 namespace {
 
 #ifndef MDN_WALK_THREADS
-#define MDN_WALK_THREADS 512
+#define MDN_WALK_THREADS 512    // 2-D slices
+#endif
+#ifndef MDN_WALK_THREADS_3D
+#define MDN_WALK_THREADS_3D 384  // 3-D grids (the unrolled walk needs more registers)
 #endif
 #ifndef MDN_WALK_MINB
 #define MDN_WALK_MINB 2
 #endif
 constexpr int kThreads = 256;
-constexpr int kWalkThreads = MDN_WALK_THREADS;
+constexpr int walk_threads(bool k3D) { return k3D ? MDN_WALK_THREADS_3D : MDN_WALK_THREADS; }
 constexpr unsigned kFull = 0xffffffffu;
 
 __device__ __forceinline__ void stage_mdnorm_mats(const MatBlock& mb, double* sM, double* sC) {
@@ -64,7 +67,13 @@ __device__ __forceinline__ void flush_counter(unsigned long long* dst, unsigned 
 
 struct AtomicEmit {
   double* h;
+#ifdef MDN_EXP_NOATOMIC  // timing experiment only: keeps the value alive without the reduction
+  __device__ __forceinline__ void operator()(int b, double val) const {
+    if (val == -1.2345e300) h[b] = val;
+  }
+#else
   __device__ __forceinline__ void operator()(int b, double val) const { atomicAdd(h + b, val); }
+#endif
 };
 
 // ---------------------------------------------------------------- M1-M3: cull + compaction
@@ -206,7 +215,7 @@ mdnorm_cull_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ 
 
 // ---------------------------------------------------------------- M3-M7: balanced piece walk
 template <bool kSmemFlux, bool kStats, bool k3D>
-__global__ void __launch_bounds__(kWalkThreads, MDN_WALK_MINB)
+__global__ void __launch_bounds__(walk_threads(k3D), MDN_WALK_MINB)
 mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
   extern __shared__ double2 wsm[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -585,15 +594,16 @@ int grid_for(int64_t work, int num_sms, int per_sm, int threads = kThreads) {
 
 template <bool kSmemFlux, bool kStats, bool k3D>
 cudaError_t launch_walk(const MdnParams& p, int num_sms, cudaStream_t s) {
+  constexpr int threads = walk_threads(k3D);
   const size_t smem = (kSmemFlux ? sizeof(double2) * p.flux.n + sizeof(int) * p.flux.ntab : 0) +
-                      sizeof(int) * 32 * (kWalkThreads / 32);
+                      sizeof(int) * 32 * (threads / 32);
   auto k = mdnorm_walk_kernel<kSmemFlux, kStats, k3D>;
   cudaError_t err = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (err != cudaSuccess) return err;
   int per_sm = 0;
-  err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kWalkThreads, smem);
+  err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, threads, smem);
   if (err != cudaSuccess) return err;
-  k<<<num_sms * std::max(per_sm, 1), kWalkThreads, smem, s>>>(p);
+  k<<<num_sms * std::max(per_sm, 1), threads, smem, s>>>(p);
   return cudaGetLastError();
 }
 

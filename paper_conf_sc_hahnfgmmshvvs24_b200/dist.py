@@ -62,8 +62,13 @@ def reduce_packed(packed, group=None, dst: int | None = 0):
     import torch.distributed as dist
     if not dist.is_available() or not dist.is_initialized() or dist.get_world_size(group) == 1:
         return packed
+    buf = packed
+    if packed.is_cuda and dist.get_backend(group) == "gloo":  # gloo (CPU tests): host staging
+        buf = packed.cpu()
     if dst is None:
-        dist.all_reduce(packed, op=dist.ReduceOp.SUM, group=group)
+        dist.all_reduce(buf, op=dist.ReduceOp.SUM, group=group)
     else:
-        dist.reduce(packed, dst=dst, op=dist.ReduceOp.SUM, group=group)
+        dist.reduce(buf, dst=dst, op=dist.ReduceOp.SUM, group=group)
+    if buf is not packed:
+        packed.copy_(buf)
     return packed

@@ -1,0 +1,192 @@
+"""More GPU parity cases: flux tables off the fast path, work counters, and the N > 1 code path
+(two processes sharing one GPU, gloo reduce) -- all through the C ABI against the fp64 oracle."""
+import json
+import os
+import socket
+import subprocess
+import sys
+
+import numpy as np
+import pytest
+
+import oracle
+import synth
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def mdn():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("needs a CUDA device")
+    import paper_conf_sc_hahnfgmmshvvs24_b200 as m
+    from paper_conf_sc_hahnfgmmshvvs24_b200 import build
+    build.build()
+    return m
+
+
+def _hist(mdn, g):
+    import torch
+    torch.cuda.synchronize()
+    t = mdn.packed_histograms(g).cpu().numpy()
+    return t[: g.nbins_total].copy(), t[g.nbins_total:].copy()
+
+
+def _assert_rel(a, b, rel=1e-12):
+    assert np.array_equal(a == 0, b == 0)
+    assert np.all(np.abs(a - b) <= rel * np.abs(b))
+
+
+def _weird_flux(n=6000):
+    """Non-uniform table larger than the shared-memory limit (4096 knots): a dense cluster of 60
+    knots inside one search cell, and knots placed exactly on plane-crossing values."""
+    rng = np.random.default_rng(11)
+    k = np.sort(np.concatenate([np.linspace(1.0, 12.0, n - 64), 5.0 + 1e-5 * np.arange(1, 61),
+                                [2.5, 5.0, 7.5, 3.75]]))
+    k = np.unique(k)
+    F = np.concatenate([[0.0], np.cumsum(rng.uniform(0.1, 1.0, len(k) - 1))])
+    return k, F
+
+
+@pytest.mark.parametrize("nflux", [6000, 300])
+def test_flux_table_paths(mdn, nflux):
+    k, F = _weird_flux(nflux)
+    wl = synth.make_workload("tiny")
+    d = np.concatenate([wl.pix_dir, [[0.0, 0.0, -1.0]]])
+    s = np.concatenate([wl.solid, [1.0]])
+    lo, hi, n = [-8.0, -8.0, 0.0], [8.0, 8.0, 20.0], [16, 16, 4]
+    g = mdn.mdnorm_create_grid(0, lo, hi, n, np.eye(3))
+    mdn.mdnorm_set_instrument(g, d, s)
+    mdn.mdnorm_set_flux(g, k, F)
+    rng = np.random.default_rng(12)
+    M = np.concatenate([np.eye(3)[None], rng.normal(size=(7, 3, 3)) * 0.6])
+    c = rng.uniform(0.5, 2.0, len(M))
+    mdn.mdnorm_accumulate_matrices(g, M, c, 2.0, 9.0)
+    norm, _ = _hist(mdn, g)
+    og = oracle.Grid(lo, hi, n)
+    onorm = oracle.mdnorm(og, d, s, k, F, M, c, 2.0, 9.0)
+    assert onorm.sum() > 0
+    _assert_rel(norm, onorm)
+    ids = np.arange(len(M) * len(s))
+    nc, ns, bins, vals = mdn.mdnorm_debug_trajectories(g, M, c, 2.0, 9.0, ids, 256)
+    for t in ids:
+        m, p = divmod(int(t), len(s))
+        onc, ons, ob, ov = oracle.mdnorm_trajectory(og, d[p], s[p], k, F, M[m], c[m], 2.0, 9.0, 256)
+        assert (nc[t], ns[t]) == (onc, ons)
+        assert np.array_equal(bins[t, :ons], ob) and np.array_equal(vals[t, :ons], ov)
+
+
+def test_work_counters_match_oracle(mdn):
+    wl = synth.make_workload("corelli")
+    g = mdn.mdnorm_create_grid(0, wl.lo, wl.hi, wl.nbins, wl.W)
+    mdn.mdnorm_set_instrument(g, wl.pix_dir, wl.solid)
+    mdn.mdnorm_set_flux(g, wl.flux_k, wl.flux_F)
+    mdn.mdnorm_stats(g, 1, read=False)
+    stride = 211
+    mdn.mdnorm_accumulate(g, wl.UB, wl.R[0], wl.ops, wl.k_min, wl.k_max, 1.0, pix_stride=stride)
+    ev = synth.events_for_run(wl, 0, n=100_000)
+    import torch
+    mdn.binmd_accumulate(g, wl.UB, wl.ops, torch.from_numpy(ev).cuda())
+    st = mdn.mdnorm_stats(g, 0)
+    og = oracle.workload_grid(wl)
+    M = oracle.mdnorm_matrices(wl.R, wl.UB, wl.ops, wl.W)
+    pix = np.arange(0, wl.npix, stride)
+    hits = segs = cross = 0
+    for m in range(len(M)):
+        for p in pix:
+            if wl.solid[p] == 0:
+                continue  # masked pixels are skipped by the kernel (reading #16)
+            nc, ns, _, _ = oracle.mdnorm_trajectory(og, wl.pix_dir[p], wl.solid[p], wl.flux_k, wl.flux_F,
+                                                    M[m], 1.0, wl.k_min, wl.k_max, 1)
+            hits += nc > 0
+            cross += max(nc - 2, 0)
+            segs += ns
+    assert st["trajectories"] == len(pix) * len(M)
+    assert st["hit_trajectories"] == hits
+    assert st["crossings"] == cross
+    assert st["segments"] == segs
+    assert st["event_op_pairs"] == len(ev) * len(wl.ops)
+    inside = (oracle.binmd_bins(og, oracle.binmd_matrices(wl.UB, wl.ops, wl.W), ev) >= 0).sum()
+    assert st["event_op_inside"] == inside
+
+
+def _free_port():
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def _dist_worker(rank, world, port, q):
+    import torch
+    import torch.distributed as dist
+    sys.path.insert(0, ROOT)
+    import paper_conf_sc_hahnfgmmshvvs24_b200 as m
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    wl = synth.make_workload("corelli", events_per_run=400_000)
+    ev = synth.events_for_run(wl, 0)
+    plan = m.plan_shards(world, rank, 1, wl.npix, len(ev))
+    g = m.mdnorm_create_grid(0, wl.lo, wl.hi, wl.nbins, wl.W)
+    m.mdnorm_set_instrument(g, wl.pix_dir, wl.solid)
+    m.mdnorm_set_flux(g, wl.flux_k, wl.flux_F)
+    m.mdnorm_accumulate(g, wl.UB, wl.R[0], wl.ops, wl.k_min, wl.k_max, 1.0,
+                        pix_begin=plan.pix_begin, pix_stride=plan.pix_stride * 13)
+    b, e = plan.event_ranges[0]
+    m.binmd_accumulate(g, wl.UB, wl.ops, torch.from_numpy(ev[b:e]).cuda())
+    packed = m.packed_histograms(g)
+    m.reduce_packed(packed, dst=0)
+    if rank == 0:
+        xs = m.mdnorm_cross_section(g)
+        torch.cuda.synchronize()
+        q.put((packed.cpu().numpy(), xs))
+    dist.barrier()
+    g.close()
+    dist.destroy_process_group()
+
+
+def test_two_processes_one_gpu_reduce(mdn):
+    """N > 1 path on real kernels: plan_shards + per-rank library histograms + one reduce; the
+    pixel stride 2*13 of the two ranks covers every 13th pixel exactly once."""
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_dist_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    packed, xs = q.get(timeout=600)
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    wl = synth.make_workload("corelli", events_per_run=400_000)
+    ev = synth.events_for_run(wl, 0)
+    og = oracle.workload_grid(wl)
+    M = oracle.mdnorm_matrices(wl.R, wl.UB, wl.ops, wl.W)
+    onorm = oracle.Accumulator(og.nbins)
+    for r in range(2):
+        oracle.mdnorm(og, wl.pix_dir, wl.solid, wl.flux_k, wl.flux_F, M, 1.0, wl.k_min, wl.k_max,
+                      pix_begin=r, pix_stride=26, acc=onorm)
+    obm = oracle.binmd(og, oracle.binmd_matrices(wl.UB, wl.ops, wl.W), ev)
+    n = og.nbins
+    _assert_rel(packed[:n], onorm.value())
+    _assert_rel(packed[n:], obm)
+    oxs = oracle.cross_section(obm, onorm.value())
+    assert np.array_equal(np.isnan(xs), np.isnan(oxs))
+
+
+def test_bench_multi_rank_code_path():
+    """bench.py under torchrun with 2 ranks (gloo, both on GPU 0): the N > 1 code path runs and
+    rank 0 prints one JSON line with n_gpus = 2 (a code-path check, not a performance number)."""
+    env = dict(os.environ, MDN_BENCH_SHARED_GPU="1")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
+           "--master-addr", "127.0.0.1", "--master-port", str(_free_port()), os.path.join(ROOT, "bench.py"),
+           "--gpus", "2", "--steps", "2", "--warmup", "1", "--no-cpu-baseline", "--dist-backend", "gloo"]
+    r = subprocess.run(cmd, env=env, capture_output=True, text=True, timeout=900, cwd=ROOT)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["scaling"] == "weak" and d["value"] > 0
+    assert d["config"]["trajectories_per_gpu"] == 372736 * 24
