@@ -273,10 +273,10 @@ mdn_status binmd_host_stream(mdn_grid* g, const MatBlock& mb, int64_t nevents, c
       MDN_CUDA(cudaEventCreateWithFlags(&g->ev_free[i], cudaEventDisableTiming), "event");
     }
   }
-  // the first copy may not run ahead of earlier work on the caller's stream that uses staging
-  for (int i = 0; i < 2; ++i) {
-    MDN_CUDA(cudaEventRecord(g->ev_free[i], s), "event record");
-  }
+  // A slot may be refilled once the last kernel that read it is done: ev_free[slot] is recorded
+  // after every scatter launch (never-recorded events are complete).  Nothing else orders the
+  // copies after earlier work on the caller's stream, so the first chunks' H2D overlaps the
+  // MDNorm kernels enqueued before this call.
   int64_t c = 0;
   for (int64_t off = 0; off < nevents; off += chunk, ++c) {
     const int slot = (int)(c & 1);
@@ -425,13 +425,15 @@ mdn_status mdnorm_set_flux(mdn_grid* g, int64_t n, const double* k, const double
     if (!(hk[i] > hk[i - 1])) return fail(MDN_EINVAL, "flux k not strictly increasing at %lld", (long long)i);
     if (hF[i] < hF[i - 1]) return fail(MDN_EINVAL, "cumulative flux F decreases at %lld", (long long)i);
   }
-  // (kappa_i, Phi_i) interleaved, plus the search start table of flux_at (M5): 2n uniform cells
-  std::vector<double2> kf((size_t)n);
+  // (kappa_i, Phi_i) interleaved + two (+inf, +inf) pads, plus the cell table of flux_at (M5):
+  // 4n uniform cells for tables staged in shared memory (uint16 copy), 2n otherwise
+  std::vector<double2> kf((size_t)n + 2);
   for (int64_t i = 0; i < n; ++i) kf[i] = make_double2(hk[i], hF[i]);
-  const int ntab = (int)std::min<int64_t>(2 * n, 1 << 22);
+  kf[n] = kf[n + 1] = make_double2(HUGE_VAL, HUGE_VAL);
+  const int ntab = (int)std::min<int64_t>((n <= mdn::kFluxSmemMax ? 4 : 2) * n, 1 << 22);
   const double cell = (hk[n - 1] - hk[0]) / (double)ntab;
-  // tab[c] = max{i : kappa_i <= fl(kappa_0 + c * cell)} (exact comparisons); the search window
-  // of a query in cell c is [tab[c-1], tab[c+2] + 1] (flux_at), nsteps bisections close it
+  // tab[c] = max{i : kappa_i <= fl(kappa_0 + c * cell)} (exact comparisons, capped at n - 2),
+  // flagged dense when cell c holds more than three knots (tab[c+1] - tab[c] > 3)
   std::vector<int> htab((size_t)ntab);
   for (int c = 0, i = 0; c < ntab; ++c) {
     const double x = hk[0] + (double)c * cell;
@@ -444,13 +446,17 @@ mdn_status mdnorm_set_flux(mdn_grid* g, int64_t n, const double* k, const double
     const int hi = c + 2 < ntab ? htab[c + 2] + 1 : (int)n - 1;
     wmax = std::max(wmax, hi - lo);
   }
+  for (int c = 0; c < ntab; ++c) {
+    const bool dense = c + 1 >= ntab || (htab[c + 1] & (int)(mdn::kFluxDense32 - 1)) - htab[c] > 3;
+    if (dense) htab[c] |= (int)mdn::kFluxDense32;
+  }
   int nsteps = 0;
   while ((1 << nsteps) < wmax) ++nsteps;
   double2* d = nullptr;
   int* tab = nullptr;
-  cudaError_t e = cudaMalloc(&d, sizeof(double2) * n);
+  cudaError_t e = cudaMalloc(&d, sizeof(double2) * (n + 2));
   if (e == cudaSuccess) e = cudaMalloc(&tab, sizeof(int) * ntab);
-  if (e == cudaSuccess) e = cudaMemcpy(d, kf.data(), sizeof(double2) * n, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemcpy(d, kf.data(), sizeof(double2) * (n + 2), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(tab, htab.data(), sizeof(int) * ntab, cudaMemcpyHostToDevice);
   if (e != cudaSuccess) {
     cudaFree(d);

@@ -99,46 +99,61 @@ __device__ __forceinline__ bool compose_binmd(const double* UB, const double* S,
 // ------------------------------------------------------------------------------ M5 flux
 // F(x): clamp outside, else i = max{i : kappa_i <= x} and
 //   Phi_i + (Phi_{i+1} - Phi_i) * ((x - kappa_i) / (kappa_{i+1} - kappa_i)).
-// i is unique, so it may be found by any search.  Here a uniform-cell table narrows it to a
-// window: tab[c] = max{i : kappa_i <= fl(kappa_0 + c * cell)} (host, exact comparisons).  The
-// cell c of x is computed approximately (off by at most one cell), so the window
-// [tab[c-1], tab[c+2] + 1] always satisfies kappa_lo <= x < kappa_hi; a fixed number of
-// branch-free bisection steps (nsteps = ceil(log2(max window)), warp-uniform) then lands on i.
+// i is unique, so it may be found by any search.  A uniform-cell table gives
+// tab[c] = max{i : kappa_i <= fl(kappa_0 + c * cell)} (host, exact comparisons), with flag bit
+// kFluxDense set when cell c holds more than 3 knots.  The cell of x is computed from an
+// approximate u (relative error ~1e-16, i.e. ~1e-12 cells); unless u is within 1e-9 of a cell
+// boundary it is exact, so for a non-dense interior cell i is tab[c] + (#probes of the next three
+// knots that are <= x) -- independent loads, no bisection, no clamps (kappa_0 < x < kappa_{n-1}
+// there).  Everything else (cell edges, dense cells, x outside the table) takes the general
+// path: the window [tab[c-1], tab[c+2] + 1] and a scan.  The knot array is padded with two
+// (+inf, +inf) entries so the probes never read out of bounds.
+constexpr unsigned kFluxDense32 = 1u << 30;  // flag bit in an int32 table entry
+constexpr unsigned kFluxDense16 = 1u << 15;  // flag bit in a uint16 (shared-memory) entry
+
 struct FluxView {
-  const double2* kf;  // (kappa_i, Phi_i)
-  const int* tab;     // ntab cell start indices
+  const double2* kf;  // (kappa_i, Phi_i), n entries + 2 padding entries
+  const void* tab;    // ntab entries: int32 (global) or uint16 (shared-memory copy)
   double k_first, F_first, k_last, F_last, inv_cell;
   int n, ntab, nsteps, pad;
 };
 
+template <typename TabT>
+__device__ __forceinline__ unsigned tab_entry(const FluxView& f, int c) {
+  return (unsigned)static_cast<const TabT*>(f.tab)[c];
+}
+
+template <typename TabT>
+__device__ __forceinline__ double flux_general(const FluxView& f, double x) {
+  constexpr unsigned flag = sizeof(TabT) == 2 ? kFluxDense16 : kFluxDense32;
+  if (x <= f.k_first) return f.F_first;
+  if (x >= f.k_last) return f.F_last;
+  const double u = fmin(fmax((x - f.k_first) * f.inv_cell, 0.0), (double)(f.ntab - 1));
+  const int c = (int)u;  // within one cell of the true cell
+  const int lo = (int)(tab_entry<TabT>(f, max(c - 1, 0)) & (flag - 1));
+  const int hi = c + 2 < f.ntab ? (int)(tab_entry<TabT>(f, c + 2) & (flag - 1)) + 1 : f.n - 1;
+  int i = lo;  // kappa_lo <= x < kappa_hi
+  while (i + 1 < hi && f.kf[i + 1].x <= x) ++i;
+  const double2 a = f.kf[i], b = f.kf[i + 1];
+  return dadd(a.y, dmul(dsub(b.y, a.y), ddiv(dsub(x, a.x), dsub(b.x, a.x))));
+}
+
+template <typename TabT = int>
 __device__ __forceinline__ double flux_at(const FluxView& f, double x) {
 #ifdef MDN_EXP_NOFLUX  // timing experiment only (wrong results): F(x) = x
   return x;
 #endif
-  // Cell of x from an approximate u (relative error ~1e-16, i.e. ~1e-12 cells): unless u is
-  // within 1e-9 of a cell boundary the cell c is exact and the window is [tab[c], tab[c+1] + 1]
-  // (the knots of one cell); near a boundary it is widened by one cell on each side.
-  const double u = fmin(fmax((x - f.k_first) * f.inv_cell, 0.0), (double)(f.ntab - 1));
-  const double cf = floor(u);
-  const int c = (int)cf;
-  const double fr = u - cf;
-  const bool edge = fr < 1e-9 || fr > 1.0 - 1e-9;
-  const int lo = f.tab[edge ? max(c - 1, 0) : c];
-  const int ch = edge ? c + 2 : c + 1;
-  const int hi = ch < f.ntab ? f.tab[ch] + 1 : f.n - 1;
-  // invariant kappa_lo <= x < kappa_hi; i = lo + #{t >= 1 : kappa_{lo+t} <= x}: three
-  // independent probes cover a cell of up to 3 knots, the loop finishes denser cells
-  int i = lo;
-#pragma unroll
-  for (int t = 1; t <= 3; ++t) {
-    const int j = lo + t;
-    if (j < hi) i += f.kf[j].x <= x ? 1 : 0;
-  }
-  if (i == lo + 3)
-    while (i + 1 < hi && f.kf[i + 1].x <= x) ++i;
+  constexpr unsigned flag = sizeof(TabT) == 2 ? kFluxDense16 : kFluxDense32;
+  const double u = (x - f.k_first) * f.inv_cell;
+  const double uf = floor(u);
+  const double fr = u - uf;
+  const bool interior = uf >= 0.0 && uf < (double)(f.ntab - 1) && fr > 1e-9 && fr < 1.0 - 1e-9;
+  const unsigned e = interior ? tab_entry<TabT>(f, (int)uf) : flag;
+  if (e & flag) return flux_general<TabT>(f, x);
+  const int i = (int)e + (f.kf[e + 1].x <= x ? 1 : 0) + (f.kf[e + 2].x <= x ? 1 : 0) +
+                (f.kf[e + 3].x <= x ? 1 : 0);
   const double2 a = f.kf[i], b = f.kf[i + 1];
-  const double F = dadd(a.y, dmul(dsub(b.y, a.y), ddiv(dsub(x, a.x), dsub(b.x, a.x))));
-  return x <= f.k_first ? f.F_first : (x >= f.k_last ? f.F_last : F);
+  return dadd(a.y, dmul(dsub(b.y, a.y), ddiv(dsub(x, a.x), dsub(b.x, a.x))));
 }
 
 // ------------------------------------------------------------------------------ M1-M2
@@ -256,7 +271,7 @@ __device__ __forceinline__ void cursor_init(AxisCursor& c, const GridC& g, int a
 // the production kernel cut long trajectories into balanced pieces.  The merge step is written
 // with selects only (no per-axis branches) so that the lanes of a warp stay converged.
 // Returns n_seg; *ncross receives the number of crossings strictly inside (lo_k, hi_k).
-template <bool k3D, class Emit>
+template <bool k3D, typename TabT = int, class Emit>
 __device__ __forceinline__ int traj_walk(const GridC& g, const FluxView& fx, double v0, double v1,
                                          double v2, double lo_k, double hi_k, double omega_c,
                                          Emit& emit, int* ncross) {
@@ -273,7 +288,7 @@ __device__ __forceinline__ int traj_walk(const GridC& g, const FluxView& fx, dou
   }
   const int total = c0.cnt + c1.cnt + c2.cnt;
   *ncross = total;
-  double k1 = lo_k, F1 = flux_at(fx, lo_k);
+  double k1 = lo_k, F1 = flux_at<TabT>(fx, lo_k);
   int nseg = 0;
   int left = total;
   // next entry of L: the smallest pending crossing (ties: lowest axis first; equal values give
@@ -336,15 +351,15 @@ __device__ __forceinline__ int traj_walk(const GridC& g, const FluxView& fx, dou
     for (; rem >= 2; rem -= 2) {
       const double ka = next();
       const double kb = next();
-      const double Fa = flux_at(fx, ka);
-      const double Fb = flux_at(fx, kb);
+      const double Fa = flux_at<TabT>(fx, ka);
+      const double Fb = flux_at<TabT>(fx, kb);
       segment(ka, Fa);
       segment(kb, Fb);
     }
   }
   for (; rem >= 1; --rem) {
     const double ka = next();
-    segment(ka, flux_at(fx, ka));
+    segment(ka, flux_at<TabT>(fx, ka));
   }
   return nseg;
 }

@@ -220,12 +220,17 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
   extern __shared__ double2 wsm[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int nwarps = blockDim.x >> 5;
+  // shared layout: knots (n + 2 padded double2) | cell table (uint16) | per-warp prefix sums
   double2* sKF = wsm;
-  int* sTab = reinterpret_cast<int*>(sKF + (kSmemFlux ? p.flux.n : 0));
-  int* sPre = sTab + (kSmemFlux ? p.flux.ntab : 0);
+  uint16_t* sTab = reinterpret_cast<uint16_t*>(sKF + (kSmemFlux ? p.flux.n + 2 : 0));
+  int* sPre = reinterpret_cast<int*>(sTab + (kSmemFlux ? (p.flux.ntab + 1) & ~1 : 0));
   if (kSmemFlux) {
-    for (int i = threadIdx.x; i < p.flux.n; i += blockDim.x) sKF[i] = p.flux.kf[i];
-    for (int i = threadIdx.x; i < p.flux.ntab; i += blockDim.x) sTab[i] = p.flux.tab[i];
+    for (int i = threadIdx.x; i < p.flux.n + 2; i += blockDim.x) sKF[i] = p.flux.kf[i];
+    const int* gtab = static_cast<const int*>(p.flux.tab);
+    for (int i = threadIdx.x; i < p.flux.ntab; i += blockDim.x) {
+      const unsigned e = (unsigned)gtab[i];
+      sTab[i] = (uint16_t)((e & (kFluxDense32 - 1)) | ((e & kFluxDense32) ? kFluxDense16 : 0u));
+    }
   }
   __syncthreads();
   FluxView fx = p.flux;
@@ -277,7 +282,9 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
           if (pi < h.P - 1) hi_k = plane_k(p.g, h.A, h.jA + (pi + 1) * h.stepG, rA);
         }
         int nc;
-        const int ns = traj_walk<k3D>(p.g, fx, v0, v1, v2, lo_k, hi_k, h.oc, emit, &nc);
+        const int ns = kSmemFlux
+                           ? traj_walk<k3D, uint16_t>(p.g, fx, v0, v1, v2, lo_k, hi_k, h.oc, emit, &nc)
+                           : traj_walk<k3D, int>(p.g, fx, v0, v1, v2, lo_k, hi_k, h.oc, emit, &nc);
         if (kStats) c_seg += ns;
       }
       __syncwarp();
@@ -595,7 +602,7 @@ int grid_for(int64_t work, int num_sms, int per_sm, int threads = kThreads) {
 template <bool kSmemFlux, bool kStats, bool k3D>
 cudaError_t launch_walk(const MdnParams& p, int num_sms, cudaStream_t s) {
   constexpr int threads = walk_threads(k3D);
-  const size_t smem = (kSmemFlux ? sizeof(double2) * p.flux.n + sizeof(int) * p.flux.ntab : 0) +
+  const size_t smem = (kSmemFlux ? sizeof(double2) * (p.flux.n + 2) + sizeof(uint16_t) * ((p.flux.ntab + 1) & ~1) : 0) +
                       sizeof(int) * 32 * (threads / 32);
   auto k = mdnorm_walk_kernel<kSmemFlux, kStats, k3D>;
   cudaError_t err = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
