@@ -621,7 +621,21 @@ cudaError_t launch_cull(const MdnParams& p, const MatBlock& mb, int num_sms, cud
   auto k = mdnorm_cull_kernel<kStats>;
   cudaError_t err = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (err != cudaSuccess) return err;
-  k<<<grid_for(p.plen, num_sms, 8), kThreads, smem, s>>>(p, mb);
+  // one wave of resident CTAs (grid-stride): no tail wave of unevenly loaded blocks
+  int per_sm = 0;
+  err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kThreads, smem);
+  if (err != cudaSuccess) return err;
+  k<<<grid_for(p.plen, num_sms, std::max(per_sm, 1)), kThreads, smem, s>>>(p, mb);
+  return cudaGetLastError();
+}
+
+template <bool kPacked, bool kStats>
+cudaError_t launch_binmd_t(const BinParams& p, const MatBlock& mb, int num_sms, cudaStream_t s) {
+  auto k = binmd_kernel<kPacked, kStats>;
+  int per_sm = 0;
+  cudaError_t err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kThreads, 0);
+  if (err != cudaSuccess) return err;
+  k<<<grid_for(p.nevents, num_sms, std::max(per_sm, 1)), kThreads, 0, s>>>(p, mb);
   return cudaGetLastError();
 }
 
@@ -659,15 +673,8 @@ cudaError_t launch_binmd(const BinParams& p, const MatBlock& mb, int num_sms, cu
   if (p.nevents <= 0 || mb.nmat <= 0) return cudaSuccess;
   const bool packed = p.stride == 4 && p.col_w == 0 && p.col_q == 1 &&
                       (reinterpret_cast<uintptr_t>(p.events) & 15) == 0;
-  const int blocks = grid_for(p.nevents, num_sms, 8);
-  if (packed) {
-    if (p.stats) binmd_kernel<true, true><<<blocks, kThreads, 0, s>>>(p, mb);
-    else binmd_kernel<true, false><<<blocks, kThreads, 0, s>>>(p, mb);
-  } else {
-    if (p.stats) binmd_kernel<false, true><<<blocks, kThreads, 0, s>>>(p, mb);
-    else binmd_kernel<false, false><<<blocks, kThreads, 0, s>>>(p, mb);
-  }
-  return cudaGetLastError();
+  if (packed) return p.stats ? launch_binmd_t<true, true>(p, mb, num_sms, s) : launch_binmd_t<true, false>(p, mb, num_sms, s);
+  return p.stats ? launch_binmd_t<false, true>(p, mb, num_sms, s) : launch_binmd_t<false, false>(p, mb, num_sms, s);
 }
 
 cudaError_t launch_cross_section(const double* norm, const double* binmd, double* xs, int64_t nbins,
