@@ -12,8 +12,8 @@
 #include <cuda_runtime.h>
 #include <math_constants.h>
 
-#ifndef MDN_MERGE2D_BRANCH
-#define MDN_MERGE2D_BRANCH 0  // 2-D slices: branchy two-stream merge instead of selects
+#ifndef MDN_MERGE2D_SELECT
+#define MDN_MERGE2D_SELECT 0  // 2-D slices: select-based two-stream merge (default: branch)
 #endif
 
 namespace mdn {
@@ -297,6 +297,21 @@ __device__ __forceinline__ int traj_walk(const GridC& g, const FluxView& fx, dou
     if (left == 0) return hi_k;
     --left;
     if (!k3D) {  // 2-D slice: two streams
+#if MDN_MERGE2D_SELECT
+      const bool p0 = c0.nk <= c1.nk;
+      const double k = p0 ? c0.nk : c1.nk;
+      const double jd = p0 ? c0.jd + c0.stepd : c1.jd + c1.stepd;
+      const int cnt = (p0 ? c0.cnt : c1.cnt) - 1;
+      const double nk = cnt > 0 ? dmul(dadd(p0 ? g.lo[0] : g.lo[1], dmul(jd, p0 ? g.w[0] : g.w[1])), p0 ? c0.r : c1.r)
+                                : CUDART_INF;
+      c0.jd = p0 ? jd : c0.jd;
+      c0.cnt = p0 ? cnt : c0.cnt;
+      c0.nk = p0 ? nk : c0.nk;
+      c1.jd = p0 ? c1.jd : jd;
+      c1.cnt = p0 ? c1.cnt : cnt;
+      c1.nk = p0 ? c1.nk : nk;
+      return k;
+#else
       if (c0.nk <= c1.nk) {
         const double k = c0.nk;
         c0.jd += c0.stepd;
@@ -309,6 +324,7 @@ __device__ __forceinline__ int traj_walk(const GridC& g, const FluxView& fx, dou
       --c1.cnt;
       c1.nk = c1.cnt > 0 ? dmul(dadd(g.lo[1], dmul(c1.jd, g.w[1])), c1.r) : CUDART_INF;
       return k;
+#endif
     }
     // three streams, selects only: advance the chosen axis with one plane evaluation
     const bool s01 = c1.nk < c0.nk;
@@ -334,9 +350,11 @@ __device__ __forceinline__ int traj_walk(const GridC& g, const FluxView& fx, dou
       const double t0 = dmul(dsub(dmul(km, v0), g.lo[0]), g.s[0]);
       const double t1 = dmul(dsub(dmul(km, v1), g.lo[1]), g.s[1]);
       const double t2 = dmul(dsub(dmul(km, v2), g.lo[2]), g.s[2]);
-      if (0.0 <= t0 && t0 < g.nd[0] && 0.0 <= t1 && t1 < g.nd[1] && 0.0 <= t2 && t2 < g.nd[2]) {
-        const int b = __double2int_rz(t0) + g.n[0] * (__double2int_rz(t1) + g.n[1] * __double2int_rz(t2));
-        emit(b, dmul(dsub(F2, F1), omega_c));
+      // for finite t, (0 <= t < n) <=> (unsigned)floor(t) < n (floor saturates, -0 -> 0); the
+      // walk only sees finite v (the cull drops non-finite directions)
+      const int i0 = __double2int_rd(t0), i1 = __double2int_rd(t1), i2 = __double2int_rd(t2);
+      if ((unsigned)i0 < (unsigned)g.n[0] && (unsigned)i1 < (unsigned)g.n[1] && (unsigned)i2 < (unsigned)g.n[2]) {
+        emit(i0 + g.n[0] * (i1 + g.n[1] * i2), dmul(dsub(F2, F1), omega_c));
         ++nseg;
       }
       k1 = k2;

@@ -135,7 +135,8 @@ mdnorm_cull_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ 
         const double v2 = row_dot(M + 6, px.x, px.y, px.z);
         const double vv[3] = {v0, v1, v2};
         double kin, kout;
-        if (traj_clip(p.g, vv, p.kmin, p.kmax, kin, kout)) {
+        // a non-finite v (only from a singular composition) contributes nothing in the oracle
+        if (isfinite(v0) && isfinite(v1) && isfinite(v2) && traj_clip(p.g, vv, p.kmin, p.kmax, kin, kout)) {
           hit = true;
           const AxisStream s0 = axis_stream(p.g, 0, v0, v0 != 0.0 ? ddiv(1.0, v0) : 0.0, kin, kout);
           const AxisStream s1 = axis_stream(p.g, 1, v1, v1 != 0.0 ? ddiv(1.0, v1) : 0.0, kin, kout);
