@@ -27,8 +27,9 @@
  *  - Ownership: the caller owns every input.  set_* calls copy their (host or device) inputs
  *    into library-owned device memory and may be freed on return.  The histograms are
  *    library-owned; mdnorm_histograms() returns borrowed device pointers valid until
- *    mdnorm_destroy().  binmd_dev == norm_dev + nbins_total always (one packed fp64 buffer
- *    [norm | binmd], so one collective covers both).
+ *    mdnorm_destroy().  The grid owns ONE packed fp64 buffer [norm | binmd | err2] of
+ *    3 * nbins_total doubles: binmd_dev == norm_dev + nbins_total and err2_dev == binmd_dev +
+ *    nbins_total always, so one collective covers all of them.
  *  - Streams: 'stream' is a cudaStream_t (NULL = legacy default stream).  Work is enqueued
  *    stream-ordered; only calls that write to a HOST pointer synchronise.  All calls on one grid
  *    must be issued on one stream, or be ordered by the caller.
@@ -79,6 +80,12 @@ mdn_status mdnorm_destroy(mdn_grid *g);
  * solid: double[npix] solid angle x vanadium factor, >= 0, 0 == masked pixel. */
 mdn_status mdnorm_set_instrument(mdn_grid *g, int64_t npix, const double *dir, const double *solid);
 
+/* Per-pixel momentum limits (Mantid's MDNorm_low/high): pixel p's
+ * trajectory then runs over [max(k_min, kmin[p]), min(k_max, kmax[p])] in every later
+ * mdnorm_accumulate*.  kmin, kmax: double[npix] (host or device), npix must equal the
+ * instrument's; kmin == kmax == NULL removes the limits.  set_instrument also removes them. */
+mdn_status mdnorm_set_pixel_krange(mdn_grid *g, int64_t npix, const double *kmin, const double *kmax);
+
 /* Integrated (cumulative) flux table F(k) (FluxFile; linear_interpolation):
  * k: double[n] strictly increasing, 1/Angstrom; F: double[n] non-decreasing; n >= 2.
  * F is clamped to F[0] below k[0] and to F[n-1] above k[n-1]. */
@@ -108,14 +115,29 @@ mdn_status binmd_accumulate(mdn_grid *g, const double UB[9], int32_t nops, const
                             int64_t nevents, const float *events, int64_t stride_floats,
                             int32_t col_w, int32_t col_q, void *stream);
 
+/* BinMD that also accumulates the error-squared column (Mantid MDEvent signal + error^2; the
+ * paper's 8-column rows): err2[b] += events[e*stride + col_e] for every (op, event)
+ * inside the grid, besides binmd[b] += weight.  col_e = -1 is plain binmd_accumulate. */
+mdn_status binmd_accumulate_err(mdn_grid *g, const double UB[9], int32_t nops, const double *ops,
+                                int64_t nevents, const float *events, int64_t stride_floats,
+                                int32_t col_w, int32_t col_e, int32_t col_q, void *stream);
+
 /* Borrowed device pointers to the fp64 histograms (each nbins_total doubles). */
 mdn_status mdnorm_histograms(mdn_grid *g, void **norm_dev, void **binmd_dev, int64_t *nbins_total);
+
+/* Borrowed device pointer to the error-squared histogram (== binmd_dev + nbins_total). */
+mdn_status mdnorm_error_histogram(mdn_grid *g, void **err2_dev);
 
 /* xs[b] = binmd[b] / norm[b] (NaN where norm[b] == 0) into xs (double[nbins_total], host or
  * device).  A host xs synchronises the stream before returning. */
 mdn_status mdnorm_cross_section(mdn_grid *g, double *xs, void *stream);
 
-/* Zero both histograms (stream-ordered). */
+/* Cross-section and its error: xs as above and xs_err[b] = sqrt(err2[b]) / norm[b] (the
+ * normalization is computed, so it carries no error; NaN where norm[b] == 0).  xs and xs_err
+ * are both host or both device arrays of nbins_total doubles. */
+mdn_status mdnorm_cross_section_err(mdn_grid *g, double *xs, double *xs_err, void *stream);
+
+/* Zero all histograms (stream-ordered). */
 mdn_status mdnorm_reset(mdn_grid *g, void *stream);
 
 /* Work counters (tracing).  enable = 1 turns counting on for later kernels, 0 turns it off,

@@ -62,6 +62,12 @@ def lib():
         _lib.orc_binmd.restype = i64
         _lib.orc_binmd_bins.argtypes = [P, i32, P, i64, P, i64, i32, i32, P]
         _lib.orc_cross_section.argtypes = [i64, P, P, P]
+        _lib.orc_mdnorm_krange.argtypes = [P, i64, P, P, P, P, i64, P, P, i32, P, P, d, d, i64, i64, i64,
+                                           P, P]
+        _lib.orc_mdnorm_krange.restype = i64
+        _lib.orc_binmd_err.argtypes = [P, i32, P, i64, P, i64, i32, i32, P, P]
+        _lib.orc_binmd_err.restype = i64
+        _lib.orc_cross_section_err.argtypes = [i64, P, P, P]
     return _lib
 
 
@@ -143,6 +149,41 @@ def mdnorm(grid: Grid, pix_dir, solid, fk, fF, M, charge, k_min, k_max,
                      _p(charge), float(k_min), float(k_max), int(pix_begin), int(pix_end),
                      int(pix_stride), _p(acc.sum), _p(acc.comp))
     return acc.value()
+
+
+def mdnorm_krange(grid: Grid, pix_dir, solid, pix_kmin, pix_kmax, fk, fF, M, charge, k_min, k_max,
+                  pix_begin=0, pix_end=None, pix_stride=1, acc: Accumulator | None = None) -> np.ndarray:
+    """mdnorm with per-pixel momentum limits (None = no limit on that side)."""
+    d, s, fk, fF = _f64(pix_dir), _f64(solid), _f64(fk), _f64(fF)
+    lo = None if pix_kmin is None else _f64(pix_kmin)
+    hi = None if pix_kmax is None else _f64(pix_kmax)
+    M = _f64(M).reshape(-1, 9)
+    charge = _f64(np.broadcast_to(np.asarray(charge, dtype=np.float64), (len(M),)))
+    acc = acc or Accumulator(grid.nbins)
+    pix_end = len(s) if pix_end is None else pix_end
+    lib().orc_mdnorm_krange(grid.ref, len(s), _p(d), _p(s), None if lo is None else _p(lo),
+                            None if hi is None else _p(hi), len(fk), _p(fk), _p(fF), len(M), _p(M),
+                            _p(charge), float(k_min), float(k_max), int(pix_begin), int(pix_end),
+                            int(pix_stride), _p(acc.sum), _p(acc.comp))
+    return acc.value()
+
+
+def binmd_err(grid: Grid, N, events, stride=None, col_e=1, col_q=5,
+              acc: Accumulator | None = None) -> np.ndarray:
+    """error-squared histogram from column col_e."""
+    ev, n, stride = _events(events, stride, col_e, col_q)
+    N = _f64(N).reshape(-1, 9)
+    acc = acc or Accumulator(grid.nbins)
+    lib().orc_binmd_err(grid.ref, len(N), _p(N), n, _p(ev), stride, col_e, col_q, _p(acc.sum),
+                        _p(acc.comp))
+    return acc.value()
+
+
+def cross_section_err(err2_h, norm_h) -> np.ndarray:
+    e, n = _f64(err2_h), _f64(norm_h)
+    out = np.empty_like(e)
+    lib().orc_cross_section_err(len(e), _p(e), _p(n), _p(out))
+    return out
 
 
 def mdnorm_trajectory(grid: Grid, d, solid, fk, fF, M, charge, k_min, k_max, max_segs=4096):

@@ -230,6 +230,19 @@ int64_t orc_mdnorm(const orc_grid *g, int64_t npix, const double *dir, const dou
                    double k_min, double k_max,
                    int64_t pix_begin, int64_t pix_end, int64_t pix_stride,
                    double *norm_sum, double *norm_comp) {
+  return orc_mdnorm_krange(g, npix, dir, solid, NULL, NULL, nflux, fk, fF, nmat, M, charge, k_min,
+                           k_max, pix_begin, pix_end, pix_stride, norm_sum, norm_comp);
+}
+
+/* Same, with optional per-pixel momentum limits (S§8(f) NEXT #1; Mantid's MDNorm_low/high):
+ * pixel p's trajectory runs over [max(k_min, pix_kmin[p]), min(k_max, pix_kmax[p])]. */
+int64_t orc_mdnorm_krange(const orc_grid *g, int64_t npix, const double *dir, const double *solid,
+                          const double *pix_kmin, const double *pix_kmax,
+                          int64_t nflux, const double *fk, const double *fF,
+                          int32_t nmat, const double *M, const double *charge,
+                          double k_min, double k_max,
+                          int64_t pix_begin, int64_t pix_end, int64_t pix_stride,
+                          double *norm_sum, double *norm_comp) {
   gconst c;
   grid_consts(g, &c);
   if (pix_end > npix) pix_end = npix;
@@ -238,8 +251,11 @@ int64_t orc_mdnorm(const orc_grid *g, int64_t npix, const double *dir, const dou
   for (int32_t m = 0; m < nmat; ++m) {
     for (int64_t p = pix_begin; p < pix_end; p += pix_stride) {
       int32_t ncross;
-      trajectory(&c, dir + 3 * p, solid[p] * charge[m], nflux, fk, fF, M + 9 * m, k_min, k_max,
-                 buf, &ncross, NULL, NULL, 0, norm_sum, norm_comp);
+      double lo = k_min, hi = k_max;
+      if (pix_kmin && pix_kmin[p] > lo) lo = pix_kmin[p];
+      if (pix_kmax && pix_kmax[p] < hi) hi = pix_kmax[p];
+      trajectory(&c, dir + 3 * p, solid[p] * charge[m], nflux, fk, fF, M + 9 * m, lo, hi, buf,
+                 &ncross, NULL, NULL, 0, norm_sum, norm_comp);
       ++ntraj;
     }
   }
@@ -290,7 +306,33 @@ void orc_binmd_bins(const orc_grid *g, int32_t nmat, const double *N, int64_t ne
       bins[m * nevents + e] = event_bin(&c, N + 9 * m, events + e * stride, col_q);
 }
 
+/* Error histogram (S§8(f) NEXT #1: Mantid's MDEvent carries signal and error squared, P:188's
+ * 8 columns): err2[b] += events[e*stride + col_e] for every (op, event) inside the grid. */
+int64_t orc_binmd_err(const orc_grid *g, int32_t nmat, const double *N, int64_t nevents,
+                      const float *events, int64_t stride, int32_t col_e, int32_t col_q,
+                      double *err_sum, double *err_comp) {
+  gconst c;
+  grid_consts(g, &c);
+  int64_t inside = 0;
+  for (int32_t m = 0; m < nmat; ++m)
+    for (int64_t e = 0; e < nevents; ++e) {
+      const float *ev = events + e * stride;
+      int64_t b = event_bin(&c, N + 9 * m, ev, col_q);
+      if (b >= 0) {
+        neu_add(err_sum, err_comp, b, (double)ev[col_e]);
+        ++inside;
+      }
+    }
+  return inside;
+}
+
 /* ------------------------------------------------------------------ X2: divide             */
 void orc_cross_section(int64_t nbins, const double *binmd, const double *norm, double *xs) {
   for (int64_t b = 0; b < nbins; ++b) xs[b] = norm[b] > 0.0 ? binmd[b] / norm[b] : NAN;
+}
+
+/* Error of the cross-section: the normalization carries no error (it is computed, not
+ * counted), so sigma_xs = sqrt(err2) / norm; NaN where norm == 0. */
+void orc_cross_section_err(int64_t nbins, const double *err2, const double *norm, double *xs_err) {
+  for (int64_t b = 0; b < nbins; ++b) xs_err[b] = norm[b] > 0.0 ? sqrt(err2[b]) / norm[b] : NAN;
 }

@@ -52,6 +52,16 @@ int64_t orc_mdnorm(const orc_grid *g, int64_t npix, const double *dir, const dou
                    int64_t pix_begin, int64_t pix_end, int64_t pix_stride,
                    double *norm_sum, double *norm_comp);
 
+/* orc_mdnorm with optional per-pixel momentum limits (NULL = none): pixel p runs over
+ * [max(k_min, pix_kmin[p]), min(k_max, pix_kmax[p])] (S§8(f) NEXT #1, Mantid MDNorm_low/high). */
+int64_t orc_mdnorm_krange(const orc_grid *g, int64_t npix, const double *dir, const double *solid,
+                          const double *pix_kmin, const double *pix_kmax,
+                          int64_t nflux, const double *fk, const double *fF,
+                          int32_t nmat, const double *M, const double *charge,
+                          double k_min, double k_max,
+                          int64_t pix_begin, int64_t pix_end, int64_t pix_stride,
+                          double *norm_sum, double *norm_comp);
+
 /* One trajectory, for bit-exact debug checks: n_cross = |L| (endpoints + kept crossings),
  * n_seg = number of segments appended, seg_bins/seg_vals = the first max_segs of them in order.
  * Returns n_seg. */
@@ -72,8 +82,16 @@ void orc_binmd_bins(const orc_grid *g, int32_t nmat, const double *N, int64_t ne
                     const float *events, int64_t stride, int32_t col_w, int32_t col_q,
                     int64_t *bins);
 
+/* Error-squared histogram: err2[b] += events[e*stride + col_e] per (op, event) inside. */
+int64_t orc_binmd_err(const orc_grid *g, int32_t nmat, const double *N, int64_t nevents,
+                      const float *events, int64_t stride, int32_t col_e, int32_t col_q,
+                      double *err_sum, double *err_comp);
+
 /* xs[b] = binmd[b] / norm[b] if norm[b] > 0 else NaN. */
 void orc_cross_section(int64_t nbins, const double *binmd, const double *norm, double *xs);
+
+/* xs_err[b] = sqrt(err2[b]) / norm[b] if norm[b] > 0 else NaN. */
+void orc_cross_section_err(int64_t nbins, const double *err2, const double *norm, double *xs_err);
 
 #ifdef __cplusplus
 }

@@ -33,6 +33,10 @@ SIGNATURES = {
     "mdnorm_histograms": [P, P, P, P],
     "mdnorm_cross_section": [P, P, P],
     "mdnorm_reset": [P, P],
+    "mdnorm_set_pixel_krange": [P, i64, P, P],
+    "binmd_accumulate_err": [P, P, i32, P, i64, P, i64, i32, i32, i32, P],
+    "mdnorm_error_histogram": [P, P],
+    "mdnorm_cross_section_err": [P, P, P, P],
     "mdnorm_stats": [P, C.c_int, P],
     "mdn_last_error": [],
     "mdn_version": [],

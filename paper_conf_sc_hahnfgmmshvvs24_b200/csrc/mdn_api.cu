@@ -23,7 +23,8 @@ struct mdn_grid {
   GridC g{};
   double W[9]{};
   mdn_acc acc = MDN_ACC_F64;
-  double* d_hist = nullptr;  // [norm | binmd], 2 * nbins doubles
+  double* d_hist = nullptr;  // [norm | binmd | err2], 3 * nbins doubles
+  double2* d_pkr = nullptr;  // per-pixel (k_lo, k_hi) limits, or nullptr
   double4* d_pix = nullptr;
   int64_t npix = 0;
   double2* d_flux = nullptr;  // (kappa_i, Phi_i), nflux entries
@@ -168,6 +169,7 @@ mdn::MdnParams mdn_params(mdn_grid* g, double k_min, double k_max, int64_t pix_b
   mdn::MdnParams p{};
   p.g = g->g;
   p.pix = g->d_pix;
+  p.pkr = g->d_pkr;
   p.pix_begin = pix_begin;
   p.pix_stride = pix_stride;
   p.nshard = nshard;
@@ -224,29 +226,40 @@ mdn_status run_mdnorm(mdn_grid* g, mdn::MdnParams p, const MatBlock& mb, cudaStr
   return MDN_OK;
 }
 
-mdn_status check_events(int64_t nevents, const float* events, int64_t stride, int32_t col_w, int32_t col_q) {
+// Event row layout: stride floats per event; weight, error-squared (-1 = none) and Q columns.
+struct EvLayout {
+  int64_t stride;
+  int32_t col_w, col_e, col_q;
+};
+
+mdn_status check_events(int64_t nevents, const float* events, const EvLayout& L) {
   if (nevents < 0) return fail(MDN_EINVAL, "nevents < 0");
   if (nevents > 0 && !events) return fail(MDN_EINVAL, "events is NULL");
-  if (stride < 4 || col_w < 0 || col_q < 0 || col_w >= stride || col_q + 3 > stride ||
-      (col_w >= col_q && col_w < col_q + 3))
-    return fail(MDN_EINVAL, "bad event layout: stride %lld, col_w %d, col_q %d", (long long)stride, col_w, col_q);
+  const bool bad_e = L.col_e >= 0 && (L.col_e >= L.stride || L.col_e == L.col_w ||
+                                      (L.col_e >= L.col_q && L.col_e < L.col_q + 3));
+  if (L.stride < 4 || L.col_w < 0 || L.col_q < 0 || L.col_e < -1 || L.col_w >= L.stride ||
+      L.col_q + 3 > L.stride || (L.col_w >= L.col_q && L.col_w < L.col_q + 3) || bad_e)
+    return fail(MDN_EINVAL, "bad event layout: stride %lld, col_w %d, col_e %d, col_q %d", (long long)L.stride,
+                L.col_w, L.col_e, L.col_q);
   return MDN_OK;
 }
 
-mdn::BinParams bin_params(mdn_grid* g, const float* ev, int64_t n, int64_t stride, int32_t col_w, int32_t col_q) {
+mdn::BinParams bin_params(mdn_grid* g, const float* ev, int64_t n, const EvLayout& L) {
   mdn::BinParams p{};
   p.g = g->g;
   p.events = ev;
   p.nevents = n;
-  p.stride = stride;
-  p.col_w = col_w;
-  p.col_q = col_q;
+  p.stride = L.stride;
+  p.col_w = L.col_w;
+  p.col_q = L.col_q;
+  p.col_e = L.col_e;
   // fp32 fast-path axis order: fewest bins first (stable), so a thin slab axis rejects early
   int ord[3] = {0, 1, 2};
   std::stable_sort(ord, ord + 3, [&](int a, int b) { return g->g.n[a] < g->g.n[b]; });
   for (int a = 0; a < 3; ++a) p.ord[a] = ord[a];
   p.acc_f32 = g->acc == MDN_ACC_F32;
   p.binmd = g->d_hist + g->g.nbins;
+  p.err2 = g->d_hist + 2 * g->g.nbins;
   p.stats = g->stats_on ? g->d_stats : nullptr;
   return p;
 }
@@ -254,12 +267,16 @@ mdn::BinParams bin_params(mdn_grid* g, const float* ev, int64_t n, int64_t strid
 // Run the BinMD kernel over host events through a two-slot staging ring: the H2D copy of chunk
 // c+1 (copy stream) overlaps the scatter of chunk c (caller's stream).
 mdn_status binmd_host_stream(mdn_grid* g, const MatBlock& mb, int64_t nevents, const float* events,
-                             int64_t stride, int32_t col_w, int32_t col_q, cudaStream_t s) {
+                             const EvLayout& L, cudaStream_t s) {
+  const int64_t stride = L.stride;
   const int64_t chunk = std::max<int64_t>(1, (int64_t)(64ll << 20) / (int64_t)(4 * stride));  // 64 MB
   const size_t need = (size_t)(chunk * stride);
   if (g->stage_floats < need) {
     for (int i = 0; i < 2; ++i) {
-      if (g->d_stage[i]) cudaFree(g->d_stage[i]);
+      if (g->d_stage[i]) {
+        cudaStreamSynchronize(s);
+        cudaFree(g->d_stage[i]);
+      }
       g->d_stage[i] = nullptr;
     }
     g->stage_floats = 0;
@@ -286,22 +303,20 @@ mdn_status binmd_host_stream(mdn_grid* g, const MatBlock& mb, int64_t nevents, c
                              cudaMemcpyHostToDevice, g->copy_stream), "H2D events");
     MDN_CUDA(cudaEventRecord(g->ev_ready[slot], g->copy_stream), "event record");
     MDN_CUDA(cudaStreamWaitEvent(s, g->ev_ready[slot], 0), "wait");
-    MDN_CUDA(mdn::launch_binmd(bin_params(g, g->d_stage[slot], n, stride, col_w, col_q), mb, g->num_sms, s),
-             "binmd kernel");
+    MDN_CUDA(mdn::launch_binmd(bin_params(g, g->d_stage[slot], n, L), mb, g->num_sms, s), "binmd kernel");
     MDN_CUDA(cudaEventRecord(g->ev_free[slot], s), "event record");
   }
   return MDN_OK;
 }
 
-mdn_status binmd_run(mdn_grid* g, const MatBlock& mb, int64_t nevents, const float* events, int64_t stride,
-                     int32_t col_w, int32_t col_q, cudaStream_t s) {
+mdn_status binmd_run(mdn_grid* g, const MatBlock& mb, int64_t nevents, const float* events, const EvLayout& L,
+                     cudaStream_t s) {
   if (nevents == 0) return ok();
   if (is_device_ptr(events)) {
-    MDN_CUDA(mdn::launch_binmd(bin_params(g, events, nevents, stride, col_w, col_q), mb, g->num_sms, s),
-             "binmd kernel");
+    MDN_CUDA(mdn::launch_binmd(bin_params(g, events, nevents, L), mb, g->num_sms, s), "binmd kernel");
     return ok();
   }
-  mdn_status st = binmd_host_stream(g, mb, nevents, events, stride, col_w, col_q, s);
+  mdn_status st = binmd_host_stream(g, mb, nevents, events, L, s);
   return st == MDN_OK ? ok() : st;
 }
 
@@ -348,8 +363,8 @@ mdn_status mdnorm_create_grid(int device, const double lo[3], const double hi[3]
   }
   g->g.nbins = total;
   std::memcpy(g->W, W, sizeof g->W);
-  e = cudaMalloc(&g->d_hist, sizeof(double) * 2 * (size_t)total);
-  if (e == cudaSuccess) e = cudaMemset(g->d_hist, 0, sizeof(double) * 2 * (size_t)total);
+  e = cudaMalloc(&g->d_hist, sizeof(double) * 3 * (size_t)total);  // [norm | binmd | err2]
+  if (e == cudaSuccess) e = cudaMemset(g->d_hist, 0, sizeof(double) * 3 * (size_t)total);
   if (e != cudaSuccess) {
     if (g->d_hist) cudaFree(g->d_hist);
     delete g;
@@ -365,6 +380,7 @@ mdn_status mdnorm_destroy(mdn_grid* g) {
   cudaDeviceSynchronize();
   cudaFree(g->d_hist);
   cudaFree(g->d_pix);
+  cudaFree(g->d_pkr);
   cudaFree(g->d_flux);
   cudaFree(g->d_ftab);
   cudaFree(g->d_hit);
@@ -408,6 +424,8 @@ mdn_status mdnorm_set_instrument(mdn_grid* g, int64_t npix, const double* dir, c
     return cuda_fail(e, "set_instrument");
   }
   cudaFree(g->d_pix);
+  cudaFree(g->d_pkr);  // per-pixel limits belong to the previous instrument
+  g->d_pkr = nullptr;
   g->d_pix = d_pix;
   g->npix = npix;
   return ok();
@@ -522,13 +540,15 @@ mdn_status mdnorm_accumulate(mdn_grid* g, const double UB[9], const double R[9],
                                 pix_stride, stream);
 }
 
-mdn_status binmd_accumulate(mdn_grid* g, const double UB[9], int32_t nops, const double* ops, int64_t nevents,
-                            const float* events, int64_t stride_floats, int32_t col_w, int32_t col_q, void* stream) {
+mdn_status binmd_accumulate_err(mdn_grid* g, const double UB[9], int32_t nops, const double* ops,
+                                int64_t nevents, const float* events, int64_t stride_floats, int32_t col_w,
+                                int32_t col_e, int32_t col_q, void* stream) {
   if (!g) return fail(MDN_EINVAL, "grid is NULL");
   mdn_status st;
+  const EvLayout L{stride_floats, col_w, col_e, col_q};
   if ((st = check_matrix(UB, "UB")) != MDN_OK) return st;
   if ((st = check_ops(nops, ops)) != MDN_OK) return st;
-  if ((st = check_events(nevents, events, stride_floats, col_w, col_q)) != MDN_OK) return st;
+  if ((st = check_events(nevents, events, L)) != MDN_OK) return st;
   DeviceGuard dg(g->device);
   MatBlock mb{};
   mb.compose = 1;
@@ -537,7 +557,12 @@ mdn_status binmd_accumulate(mdn_grid* g, const double UB[9], int32_t nops, const
   std::memcpy(mb.UB, UB, sizeof mb.UB);
   std::memcpy(mb.W, g->W, sizeof mb.W);
   std::memcpy(mb.u.c.ops, ops, sizeof(double) * 9 * nops);
-  return binmd_run(g, mb, nevents, events, stride_floats, col_w, col_q, (cudaStream_t)stream);
+  return binmd_run(g, mb, nevents, events, L, (cudaStream_t)stream);
+}
+
+mdn_status binmd_accumulate(mdn_grid* g, const double UB[9], int32_t nops, const double* ops, int64_t nevents,
+                            const float* events, int64_t stride_floats, int32_t col_w, int32_t col_q, void* stream) {
+  return binmd_accumulate_err(g, UB, nops, ops, nevents, events, stride_floats, col_w, -1, col_q, stream);
 }
 
 mdn_status mdnorm_histograms(mdn_grid* g, void** norm_dev, void** binmd_dev, int64_t* nbins_total) {
@@ -545,6 +570,70 @@ mdn_status mdnorm_histograms(mdn_grid* g, void** norm_dev, void** binmd_dev, int
   if (norm_dev) *norm_dev = g->d_hist;
   if (binmd_dev) *binmd_dev = g->d_hist + g->g.nbins;
   if (nbins_total) *nbins_total = g->g.nbins;
+  return ok();
+}
+
+mdn_status mdnorm_error_histogram(mdn_grid* g, void** err2_dev) {
+  if (!g || !err2_dev) return fail(MDN_EINVAL, "NULL argument");
+  *err2_dev = g->d_hist + 2 * g->g.nbins;
+  return ok();
+}
+
+mdn_status mdnorm_set_pixel_krange(mdn_grid* g, int64_t npix, const double* kmin, const double* kmax) {
+  if (!g) return fail(MDN_EINVAL, "grid is NULL");
+  if (!kmin && !kmax) {
+    DeviceGuard dg(g->device);
+    cudaDeviceSynchronize();
+    cudaFree(g->d_pkr);
+    g->d_pkr = nullptr;
+    return ok();
+  }
+  if (!g->d_pix) return fail(MDN_ESTATE, "mdnorm_set_instrument has not been called");
+  if (!kmin || !kmax) return fail(MDN_EINVAL, "give both kmin and kmax (or neither)");
+  if (npix != g->npix) return fail(MDN_EINVAL, "npix %lld != instrument's %lld", (long long)npix, (long long)g->npix);
+  DeviceGuard dg(g->device);
+  std::vector<double> lo, hi;
+  MDN_CUDA(to_host(kmin, npix, lo), "read kmin");
+  MDN_CUDA(to_host(kmax, npix, hi), "read kmax");
+  std::vector<double2> r((size_t)npix);
+  for (int64_t i = 0; i < npix; ++i) {
+    if (std::isnan(lo[i]) || std::isnan(hi[i])) return fail(MDN_EINVAL, "NaN momentum limit at pixel %lld", (long long)i);
+    r[i] = make_double2(lo[i], hi[i]);
+  }
+  double2* d = nullptr;
+  cudaError_t e = cudaMalloc(&d, sizeof(double2) * npix);
+  if (e == cudaSuccess) e = cudaMemcpy(d, r.data(), sizeof(double2) * npix, cudaMemcpyHostToDevice);
+  if (e != cudaSuccess) {
+    cudaFree(d);
+    return cuda_fail(e, "set_pixel_krange");
+  }
+  cudaDeviceSynchronize();
+  cudaFree(g->d_pkr);
+  g->d_pkr = d;
+  return ok();
+}
+
+mdn_status mdnorm_cross_section_err(mdn_grid* g, double* xs, double* xs_err, void* stream) {
+  if (!g) return fail(MDN_EINVAL, "grid is NULL");
+  if (!xs || !xs_err) return fail(MDN_EINVAL, "xs or xs_err is NULL");
+  const bool dx = is_device_ptr(xs), de = is_device_ptr(xs_err);
+  if (dx != de) return fail(MDN_EINVAL, "xs and xs_err must both be host or both device arrays");
+  DeviceGuard dg(g->device);
+  cudaStream_t s = (cudaStream_t)stream;
+  const int64_t n = g->g.nbins;
+  const double* h = g->d_hist;
+  if (dx) {
+    MDN_CUDA(mdn::launch_cross_section_err(h, h + n, h + 2 * n, xs, xs_err, n, g->num_sms, s), "xs kernel");
+    return ok();
+  }
+  double* d2 = nullptr;
+  MDN_CUDA(cudaMallocAsync(&d2, sizeof(double) * 2 * n, s), "xs scratch");
+  cudaError_t e = mdn::launch_cross_section_err(h, h + n, h + 2 * n, d2, d2 + n, n, g->num_sms, s);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(xs, d2, sizeof(double) * n, cudaMemcpyDeviceToHost, s);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(xs_err, d2 + n, sizeof(double) * n, cudaMemcpyDeviceToHost, s);
+  cudaFreeAsync(d2, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) return cuda_fail(e, "xs_err");
   return ok();
 }
 
@@ -568,7 +657,7 @@ mdn_status mdnorm_cross_section(mdn_grid* g, double* xs, void* stream) {
 mdn_status mdnorm_reset(mdn_grid* g, void* stream) {
   if (!g) return fail(MDN_EINVAL, "grid is NULL");
   DeviceGuard dg(g->device);
-  MDN_CUDA(cudaMemsetAsync(g->d_hist, 0, sizeof(double) * 2 * g->g.nbins, (cudaStream_t)stream), "memset");
+  MDN_CUDA(cudaMemsetAsync(g->d_hist, 0, sizeof(double) * 3 * g->g.nbins, (cudaStream_t)stream), "memset");
   if (g->d_stats) MDN_CUDA(cudaMemsetAsync(g->d_stats, 0, sizeof(unsigned long long) * 6, (cudaStream_t)stream), "memset");
   return ok();
 }
@@ -623,13 +712,13 @@ mdn_status binmd_accumulate_matrices(mdn_grid* g, int32_t nmat, const double* N,
   if (nmat < 1 || nmat > MDN_MAX_MATS || !N) return fail(MDN_EINVAL, "nmat %d outside [1, %d]", nmat, MDN_MAX_MATS);
   if (!finite_all(N, 9 * (int64_t)nmat)) return fail(MDN_EINVAL, "non-finite matrices");
   mdn_status st;
-  if ((st = check_events(nevents, events, stride_floats, col_w, col_q)) != MDN_OK) return st;
+  if ((st = check_events(nevents, events, EvLayout{stride_floats, col_w, -1, col_q})) != MDN_OK) return st;
   DeviceGuard dg(g->device);
   MatBlock mb{};
   mb.compose = 0;
   mb.nmat = nmat;
   std::memcpy(mb.u.M, N, sizeof(double) * 9 * nmat);
-  return binmd_run(g, mb, nevents, events, stride_floats, col_w, col_q, (cudaStream_t)stream);
+  return binmd_run(g, mb, nevents, events, EvLayout{stride_floats, col_w, -1, col_q}, (cudaStream_t)stream);
 }
 
 mdn_status mdnorm_debug_trajectories(mdn_grid* g, int32_t nmat, const double* M, const double* charge,
@@ -686,7 +775,7 @@ mdn_status binmd_debug_bins(mdn_grid* g, int32_t nmat, const double* N, int64_t 
   if (!g) return fail(MDN_EINVAL, "grid is NULL");
   if (nmat < 1 || nmat > MDN_MAX_MATS || !N || !bins) return fail(MDN_EINVAL, "bad debug arguments");
   mdn_status st;
-  if ((st = check_events(nevents, events, stride_floats, col_w, col_q)) != MDN_OK) return st;
+  if ((st = check_events(nevents, events, EvLayout{stride_floats, col_w, -1, col_q})) != MDN_OK) return st;
   if (nevents == 0) return ok();
   DeviceGuard dg(g->device);
   MatBlock mb{};
@@ -703,7 +792,7 @@ mdn_status binmd_debug_bins(mdn_grid* g, int32_t nmat, const double* N, int64_t 
   }
   if (e == cudaSuccess) e = cudaMalloc(&d_bins, sizeof(int64_t) * nevents * nmat);
   if (e == cudaSuccess)
-    e = mdn::launch_debug_bins(bin_params(g, dev ? events : d_ev, nevents, stride_floats, col_w, col_q), mb, d_bins,
+    e = mdn::launch_debug_bins(bin_params(g, dev ? events : d_ev, nevents, EvLayout{stride_floats, col_w, -1, col_q}), mb, d_bins,
                                nullptr);
   if (e == cudaSuccess) e = cudaDeviceSynchronize();
   if (e == cudaSuccess) e = cudaMemcpy(bins, d_bins, sizeof(int64_t) * nevents * nmat, cudaMemcpyDeviceToHost);

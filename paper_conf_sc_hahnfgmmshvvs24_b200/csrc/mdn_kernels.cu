@@ -21,7 +21,7 @@ namespace mdn {
 namespace {
 
 #ifndef MDN_WALK_THREADS
-#define MDN_WALK_THREADS 512    // 2-D slices
+#define MDN_WALK_THREADS 448    // 2-D slices (measured: 448 > 384 ~ 512 on the CORELLI slab)
 #endif
 #ifndef MDN_WALK_THREADS_3D
 #define MDN_WALK_THREADS_3D 384  // 3-D grids (the unrolled walk needs more registers)
@@ -76,6 +76,18 @@ struct AtomicEmit {
 #endif
 };
 
+// Momentum range of a pixel's trajectories: the call's [k_min, k_max], intersected with the
+// pixel's own limits when set (Mantid MDNorm_low/high; oracle orc_mdnorm_krange).
+__device__ __forceinline__ void pixel_krange(const MdnParams& p, int64_t pixel, double& lo, double& hi) {
+  lo = p.kmin;
+  hi = p.kmax;
+  if (p.pkr) {
+    const double2 r = p.pkr[pixel];
+    if (r.x > lo) lo = r.x;
+    if (r.y < hi) hi = r.y;
+  }
+}
+
 // ---------------------------------------------------------------- M1-M3: cull + compaction
 // One thread per pixel of the slab, looping over every (run, op) matrix of the launch (pixel
 // read once; matrices are warp-uniform smem broadcasts).  A conservative fp32 slab test with a
@@ -110,7 +122,6 @@ mdnorm_cull_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ 
     }
   }
   __syncthreads();
-  const float kmin32 = (float)p.kmin, kmax32 = (float)p.kmax;
   const int lane = threadIdx.x & 31;
   // per-warp ring of fp32 survivors (pixel offset, matrix); the exact fp64 path runs only when
   // 32 of them are queued, so it executes with the whole warp converged
@@ -127,7 +138,10 @@ mdnorm_cull_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ 
     if (lane < n) {
       const int slot = (qhead + lane) & 63;
       const uint32_t off = qoff[slot], m = qmat[slot];
-      const double4 px = p.pix[p.pix_begin + (int64_t)(p.p0 + off) * p.pix_stride];
+      const int64_t pixel = p.pix_begin + (int64_t)(p.p0 + off) * p.pix_stride;
+      const double4 px = p.pix[pixel];
+      double klo, khi;
+      pixel_krange(p, pixel, klo, khi);
       {
         const double* M = sM + 9 * m;
         const double v0 = row_dot(M, px.x, px.y, px.z);
@@ -136,7 +150,7 @@ mdnorm_cull_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ 
         const double vv[3] = {v0, v1, v2};
         double kin, kout;
         // a non-finite v (only from a singular composition) contributes nothing in the oracle
-        if (isfinite(v0) && isfinite(v1) && isfinite(v2) && traj_clip(p.g, vv, p.kmin, p.kmax, kin, kout)) {
+        if (isfinite(v0) && isfinite(v1) && isfinite(v2) && traj_clip(p.g, vv, klo, khi, kin, kout)) {
           hit = true;
           const AxisStream s0 = axis_stream(p.g, 0, v0, v0 != 0.0 ? ddiv(1.0, v0) : 0.0, kin, kout);
           const AxisStream s1 = axis_stream(p.g, 1, v1, v1 != 0.0 ? ddiv(1.0, v1) : 0.0, kin, kout);
@@ -182,10 +196,17 @@ mdnorm_cull_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ 
     const uint32_t off = base + lane;
     const bool valid = off < p.plen;
     double4 px = make_double4(0.0, 0.0, 0.0, 0.0);
-    if (valid) px = p.pix[p.pix_begin + (int64_t)(p.p0 + off) * p.pix_stride];
+    double klo = p.kmin, khi = p.kmax;
+    if (valid) {
+      const int64_t pixel = p.pix_begin + (int64_t)(p.p0 + off) * p.pix_stride;
+      px = p.pix[pixel];
+      pixel_krange(p, pixel, klo, khi);
+    }
     if (kStats && valid) c_traj += mb.nmat;
-    const bool live = valid && px.w != 0.0;  // masked pixels contribute 0 (reading #16)
+    // masked pixels contribute 0 (reading #16); an empty per-pixel k range contributes 0
+    const bool live = valid && px.w != 0.0 && klo < khi;
     const float q0 = (float)px.x, q1 = (float)px.y, q2 = (float)px.z;
+    const float kmin32 = (float)klo, kmax32 = (float)khi;
     for (int m = 0; m < mb.nmat; ++m) {
       const CullMat cm = sF[m];
       bool maybe = live;
@@ -309,8 +330,8 @@ struct BinAxis32 {
 // class, bin and fp64 red.add.  Out of line so that its constants are not hoisted into the
 // class-test loop.  Returns the number of (event, op) pairs that landed inside the grid.
 __device__ __noinline__ unsigned binmd_members(const BinParams& p, const double* sN, const BinAxis32* sA,
-                                               const int* sCls, const int* sMem, float4 ev, int c, int a0,
-                                               int a1) {
+                                               const int* sCls, const int* sMem, float4 ev, float e2, int c,
+                                               int a0, int a1) {
   const float w = ev.x, q0 = ev.y, q1 = ev.z, q2 = ev.w;
   const float qm = fmaxf(fabsf(q0), fmaxf(fabsf(q1), fabsf(q2)));
   const int j0 = sCls[c], j1 = sCls[c + 1];
@@ -353,6 +374,7 @@ __device__ __noinline__ unsigned binmd_members(const BinParams& p, const double*
       b = (int)be;
     }
     atomicAdd(p.binmd + b, (double)w);
+    if (p.col_e >= 0) atomicAdd(p.err2 + b, (double)e2);
     ++inside;
   }
   return inside;
@@ -422,8 +444,11 @@ binmd_kernel(const __grid_constant__ BinParams p, const __grid_constant__ MatBlo
   // only when 32 are queued, with the warp converged
   __shared__ float4 sQv[(kThreads / 32) * 64];
   __shared__ int sQc[(kThreads / 32) * 64];
+  __shared__ float sQe[(kThreads / 32) * 64];  // error-squared column (col_e >= 0 only)
   float4* qv = sQv + (threadIdx.x >> 5) * 64;
   int* qc = sQc + (threadIdx.x >> 5) * 64;
+  float* qe = sQe + (threadIdx.x >> 5) * 64;
+  const bool has_err = !kPacked && p.col_e >= 0;
   int qhead = 0, qcnt = 0;
   unsigned long long c_pairs = 0, c_in = 0;
 
@@ -432,7 +457,7 @@ binmd_kernel(const __grid_constant__ BinParams p, const __grid_constant__ MatBlo
     __syncwarp();
     if (lane < n) {
       const int slot = (qhead + lane) & 63;
-      c_in += binmd_members(p, sN, sA, sCls, sMem, qv[slot], qc[slot], a0, a1);
+      c_in += binmd_members(p, sN, sA, sCls, sMem, qv[slot], has_err ? qe[slot] : 0.0f, qc[slot], a0, a1);
     }
     qhead = (qhead + n) & 63;
     qcnt -= n;
@@ -448,12 +473,21 @@ binmd_kernel(const __grid_constant__ BinParams p, const __grid_constant__ MatBlo
 
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   int64_t base = (int64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31);  // warp-uniform
+  auto load_e = [&](int64_t e) { return has_err ? __ldcs(p.events + e * p.stride + p.col_e) : 0.0f; };
   float4 cur = make_float4(0.f, 0.f, 0.f, 0.f);
-  if (base + lane < p.nevents) cur = load(base + lane);
+  float cur_e = 0.f;
+  if (base + lane < p.nevents) {
+    cur = load(base + lane);
+    cur_e = load_e(base + lane);
+  }
   for (; base < p.nevents; base += stride) {
     const bool valid = base + lane < p.nevents;
     float4 nxt = make_float4(0.f, 0.f, 0.f, 0.f);  // software prefetch of the next event
-    if (base + stride + lane < p.nevents) nxt = load(base + stride + lane);
+    float nxt_e = 0.f;
+    if (base + stride + lane < p.nevents) {
+      nxt = load(base + stride + lane);
+      nxt_e = load_e(base + stride + lane);
+    }
     const float q0 = cur.y, q1 = cur.z, q2 = cur.w;
     const float qm = fmaxf(fabsf(q0), fmaxf(fabsf(q1), fabsf(q2)));
     if (kStats && valid) c_pairs += mb.nmat;
@@ -469,11 +503,13 @@ binmd_kernel(const __grid_constant__ BinParams p, const __grid_constant__ MatBlo
         const int slot = (qhead + qcnt + __popc(mask & ((1u << lane) - 1u))) & 63;
         qv[slot] = cur;
         qc[slot] = c;
+        if (has_err) qe[slot] = cur_e;
       }
       qcnt += __popc(mask);
       if (qcnt >= 32) drain(32);
     }
     cur = nxt;
+    cur_e = nxt_e;
   }
   if (qcnt > 0) drain(qcnt);
   if (kStats) {
@@ -490,6 +526,17 @@ xs_kernel(const double* __restrict__ norm, const double* __restrict__ binmd, dou
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
     const double d = norm[i];
     xs[i] = d > 0.0 ? ddiv(binmd[i], d) : CUDART_NAN;
+  }
+}
+
+__global__ void __launch_bounds__(kThreads)
+xs_err_kernel(const double* __restrict__ norm, const double* __restrict__ binmd, const double* __restrict__ err2,
+              double* __restrict__ xs, double* __restrict__ xs_err, int64_t n) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
+    const double d = norm[i];
+    xs[i] = d > 0.0 ? ddiv(binmd[i], d) : CUDART_NAN;
+    xs_err[i] = d > 0.0 ? ddiv(__dsqrt_rn(err2[i]), d) : CUDART_NAN;  // IEEE sqrt, as the oracle
   }
 }
 
@@ -554,8 +601,9 @@ debug_traj_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ M
   const double* M = sM + 9 * m;
   const double v[3] = {row_dot(M, px.x, px.y, px.z), row_dot(M + 3, px.x, px.y, px.z),
                        row_dot(M + 6, px.x, px.y, px.z)};
-  double kin, kout;
-  if (!traj_clip(p.g, v, p.kmin, p.kmax, kin, kout)) {
+  double kin, kout, klo, khi;
+  pixel_krange(p, pi, klo, khi);
+  if (!traj_clip(p.g, v, klo, khi, kin, kout)) {
     n_cross[t] = 0;
     n_seg[t] = 0;
     return;
@@ -681,6 +729,12 @@ cudaError_t launch_binmd(const BinParams& p, const MatBlock& mb, int num_sms, cu
 cudaError_t launch_cross_section(const double* norm, const double* binmd, double* xs, int64_t nbins,
                                  int num_sms, cudaStream_t s) {
   xs_kernel<<<grid_for(nbins, num_sms, 8), kThreads, 0, s>>>(norm, binmd, xs, nbins);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_cross_section_err(const double* norm, const double* binmd, const double* err2, double* xs,
+                                     double* xs_err, int64_t nbins, int num_sms, cudaStream_t s) {
+  xs_err_kernel<<<grid_for(nbins, num_sms, 8), kThreads, 0, s>>>(norm, binmd, err2, xs, xs_err, nbins);
   return cudaGetLastError();
 }
 

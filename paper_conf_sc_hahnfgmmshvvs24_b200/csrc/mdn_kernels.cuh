@@ -12,7 +12,7 @@ constexpr int kMaxMats = 64;          // MDN_MAX_MATS
 constexpr int kRunsPerLaunch = 16;    // runs composed per MDNorm launch (batched API)
 constexpr int kFluxSmemMax = 4096;    // flux knots staged in shared memory (64 KB of double2)
 #ifndef MDN_PIECE_SEGS
-#define MDN_PIECE_SEGS 24
+#define MDN_PIECE_SEGS 40  // measured: 40 > 24 > 16 (TOPAZ 200^3), ~flat on the CORELLI slab
 #endif
 constexpr int kPieceSegs = MDN_PIECE_SEGS;  // target segments per work piece (load balance, M4-M7)
 
@@ -54,6 +54,7 @@ struct DevCounters {
 struct MdnParams {
   GridC g;
   const double4* pix;      // (q0, q1, q2, Omega) per pixel, q = z - d  (M1)
+  const double2* pkr;      // per-pixel (k_lo, k_hi) limits, or nullptr (NEXT #1)
   int64_t pix_begin, pix_stride, nshard;
   FluxView flux;           // device pointers (global)
   int32_t acc_f32;
@@ -71,9 +72,11 @@ struct BinParams {
   const float* events;
   int64_t nevents, stride;
   int32_t col_w, col_q;
+  int32_t col_e;           // error-squared column, or -1
   int32_t ord[3];          // axis test order of the fp32 fast path (fewest bins first)
   int32_t acc_f32;
   double* binmd;           // fp64 histogram (nbins)
+  double* err2;            // fp64 error-squared histogram (nbins), used when col_e >= 0
   unsigned long long* stats;  // nullptr, or [.., .., .., .., pairs, inside] (+= per launch)
 };
 
@@ -87,6 +90,8 @@ cudaError_t launch_mdnorm(const MdnParams& p, const MatBlock& mb, int num_sms, c
 cudaError_t launch_binmd(const BinParams& p, const MatBlock& mb, int num_sms, cudaStream_t s);
 cudaError_t launch_cross_section(const double* norm, const double* binmd, double* xs, int64_t nbins,
                                  int num_sms, cudaStream_t s);
+cudaError_t launch_cross_section_err(const double* norm, const double* binmd, const double* err2, double* xs,
+                                     double* xs_err, int64_t nbins, int num_sms, cudaStream_t s);
 cudaError_t launch_debug_traj(const MdnParams& p, const MatBlock& mb, int64_t ntraj,
                               const int64_t* ids, int64_t npix, int32_t* n_cross, int32_t* n_seg,
                               int64_t* seg_bins, double* seg_vals, int64_t max_segs, cudaStream_t s);

@@ -156,6 +156,49 @@ def binmd_accumulate(g: Grid, UB, ops, events, stride_floats=None, col_w=0, col_
                                   _stream(stream, g.device)), "binmd_accumulate")
 
 
+def binmd_accumulate_err(g: Grid, UB, ops, events, stride_floats=None, col_w=0, col_e=1, col_q=5,
+                         stream=None) -> None:
+    """BinMD plus the error-squared column (8-column rows: signal 0, error^2 1, Q 5-7)."""
+    n, stride_floats = _event_layout(events, stride_floats)
+    ops = np.ascontiguousarray(ops, dtype=np.float64).reshape(-1, 9)
+    ev_p, ev_k = _arg(events, np.float32, n * stride_floats, "events")
+    UB_p, UB_k = _arg(UB, np.float64, 9)
+    check(load().binmd_accumulate_err(g.handle, UB_p, len(ops), ops.ctypes.data, n, ev_p,
+                                      int(stride_floats), int(col_w), int(col_e), int(col_q),
+                                      _stream(stream, g.device)), "binmd_accumulate_err")
+
+
+def mdnorm_set_pixel_krange(g: Grid, kmin, kmax) -> None:
+    """Per-pixel momentum limits (None, None removes them)."""
+    if kmin is None and kmax is None:
+        check(load().mdnorm_set_pixel_krange(g.handle, 0, None, None), "mdnorm_set_pixel_krange")
+        return
+    n = len(kmin)
+    lo_p, lo_k = _arg(kmin, np.float64, n, "kmin")
+    hi_p, hi_k = _arg(kmax, np.float64, n, "kmax")
+    check(load().mdnorm_set_pixel_krange(g.handle, n, lo_p, hi_p), "mdnorm_set_pixel_krange")
+
+
+def mdnorm_error_histogram(g: Grid) -> int:
+    """Borrowed device pointer of the error-squared histogram."""
+    p = C.c_void_p()
+    check(load().mdnorm_error_histogram(g.handle, C.byref(p)), "mdnorm_error_histogram")
+    return p.value
+
+
+def mdnorm_cross_section_err(g: Grid, xs=None, xs_err=None, stream=None):
+    """(xs, xs_err) as host numpy arrays (allocated if None) or CUDA tensors."""
+    if xs is None:
+        xs = np.empty(g.nbins_total, dtype=np.float64)
+    if xs_err is None:
+        xs_err = np.empty(g.nbins_total, dtype=np.float64)
+    a_p, _ = _arg(xs, np.float64, g.nbins_total, "xs")
+    b_p, _ = _arg(xs_err, np.float64, g.nbins_total, "xs_err")
+    check(load().mdnorm_cross_section_err(g.handle, a_p, b_p, _stream(stream, g.device)),
+          "mdnorm_cross_section_err")
+    return xs, xs_err
+
+
 def mdnorm_histograms(g: Grid):
     """(norm_ptr, binmd_ptr, nbins_total) -- borrowed device pointers."""
     a, b, n = C.c_void_p(), C.c_void_p(), C.c_int64()
@@ -207,11 +250,11 @@ class _CudaArray:
 
 
 def packed_histograms(g: Grid):
-    """torch float64 CUDA view of the library-owned packed [norm | binmd] buffer (2*nbins),
-    valid while g lives -- the buffer one collective reduces."""
+    """torch float64 CUDA view of the library-owned packed [norm | binmd | err2] buffer
+    (3*nbins), valid while g lives -- the buffer one collective reduces."""
     import torch
     a, _, n = mdnorm_histograms(g)
-    return torch.as_tensor(_CudaArray(a, 2 * n), device=f"cuda:{g.device}")
+    return torch.as_tensor(_CudaArray(a, 3 * n), device=f"cuda:{g.device}")
 
 
 # ------------------------------------------------------------------------------ parity entry points

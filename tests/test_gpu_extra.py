@@ -31,7 +31,8 @@ def _hist(mdn, g):
     import torch
     torch.cuda.synchronize()
     t = mdn.packed_histograms(g).cpu().numpy()
-    return t[: g.nbins_total].copy(), t[g.nbins_total:].copy()
+    n = g.nbins_total
+    return t[:n].copy(), t[n:2 * n].copy()
 
 
 def _assert_rel(a, b, rel=1e-12):
@@ -171,7 +172,7 @@ def test_two_processes_one_gpu_reduce(mdn):
     obm = oracle.binmd(og, oracle.binmd_matrices(wl.UB, wl.ops, wl.W), ev)
     n = og.nbins
     _assert_rel(packed[:n], onorm.value())
-    _assert_rel(packed[n:], obm)
+    _assert_rel(packed[n:2 * n], obm)
     oxs = oracle.cross_section(obm, onorm.value())
     assert np.array_equal(np.isnan(xs), np.isnan(oxs))
 

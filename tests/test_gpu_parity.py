@@ -39,7 +39,7 @@ def hist(mdn, g):
     torch.cuda.synchronize()
     t = mdn.packed_histograms(g).cpu().numpy()
     n = g.nbins_total
-    return t[:n].copy(), t[n:].copy()
+    return t[:n].copy(), t[n:2 * n].copy()
 
 
 def assert_rel(gpu, ref, rel=REL64, what="hist"):

@@ -397,3 +397,81 @@ def test_cross_section_nan_mask(orc):
     xs = orc.cross_section(bm, norm)
     assert np.isnan(xs[0]) and np.isnan(xs[3])
     assert xs[1] == 3.0 and xs[2] == 0.5 and xs[4] == 0.0
+
+
+# ----------------------------------------------------------------------------- NEXT #1 inputs
+
+
+def test_pixel_krange_closed_form_and_additivity(orc):
+    """Per-pixel momentum limits (Mantid MDNorm_low/high): each pixel's trajectory is clipped to
+    [max(k_min, lo_p), min(k_max, hi_p)] -- closed form on axis-aligned trajectories, identity when
+    the limits equal the global range, additivity when the range is split at k_c."""
+    rng = np.random.default_rng(21)
+    phi0 = 2.0
+    fk, fF = np.array([0.5, 30.0]), np.array([0.0, phi0 * 29.5])
+    n2, lo2, hi2 = 17, 0.5, 25.0
+    grid = orc.Grid([-1e3, -1e3, lo2], [1e3, 1e3, hi2], [1, 1, n2])
+    d = rng.normal(size=(12, 3))
+    d /= np.linalg.norm(d, axis=1)[:, None]
+    d = d[1 - d[:, 2] > 0.1]
+    s = rng.uniform(0.5, 2.0, len(d))
+    alpha = 0.8
+    kmin, kmax = 1.5, 18.0
+    plo = rng.uniform(1.0, 8.0, len(d))
+    phi = plo + rng.uniform(0.5, 9.0, len(d))
+    h = orc.mdnorm_krange(grid, d, s, plo, phi, fk, fF, (alpha * np.eye(3))[None], [1.0], kmin, kmax)
+    expect = sum(_closed_form_axis2(lo2, hi2, n2, alpha * (1 - dp[2]), max(kmin, a), min(kmax, b), sp, phi0)
+                 for dp, sp, a, b in zip(d, s, plo, phi))
+    np.testing.assert_allclose(h, expect, rtol=1e-12, atol=1e-12 * expect.max())
+    wl = synth.make_workload("corelli")
+    g2 = orc.Grid(wl.lo, wl.hi, [60, 60, 1])
+    dd, ss = wl.pix_dir[::997], wl.solid[::997]
+    M = orc.mdnorm_matrices(wl.R, wl.UB, wl.ops[:4], wl.W)
+    ones = np.ones(len(ss))
+    base = orc.mdnorm(g2, dd, ss, wl.flux_k, wl.flux_F, M, 1.0, wl.k_min, wl.k_max)
+    same = orc.mdnorm_krange(g2, dd, ss, wl.k_min * ones, wl.k_max * ones, wl.flux_k, wl.flux_F, M, 1.0,
+                             wl.k_min, wl.k_max)
+    assert np.array_equal(base, same)
+    kc = 5.3
+    lower = orc.mdnorm_krange(g2, dd, ss, None, kc * ones, wl.flux_k, wl.flux_F, M, 1.0, wl.k_min, wl.k_max)
+    upper = orc.mdnorm_krange(g2, dd, ss, kc * ones, None, wl.flux_k, wl.flux_F, M, 1.0, wl.k_min, wl.k_max)
+    np.testing.assert_allclose(lower + upper, base, rtol=1e-11, atol=1e-11 * base.max())
+    none = orc.mdnorm_krange(g2, dd, ss, 20.0 * ones, None, wl.flux_k, wl.flux_F, M, 1.0, wl.k_min, wl.k_max)
+    assert not none.any()
+
+
+def test_error_histogram_pins(orc):
+    """Error-squared histogram (8-column events: signal col 0, error^2 col 1, Q cols 5-7):
+    err2 equals the weight histogram when err^2 = w (Poisson counts); the hand example of
+    tests/golden/binmd_hand.json with err^2 = w^2 gives the squared weights; duplicating every
+    event doubles binmd and err2, so xs is unchanged and xs_err scales by 1/sqrt(2)."""
+    wl = synth.make_workload("corelli", events_per_run=30000)
+    ev = synth.events_for_run(wl, 0)
+    ev8 = np.zeros((len(ev), 8), np.float32)
+    ev8[:, 0] = ev[:, 0]
+    ev8[:, 1] = ev[:, 0]
+    ev8[:, 5:8] = ev[:, 1:4]
+    g = orc.Grid(wl.lo, wl.hi, [60, 60, 1])
+    N = orc.binmd_matrices(wl.UB, wl.ops, wl.W)
+    b = orc.binmd(g, N, ev8, col_w=0, col_q=5)
+    e2 = orc.binmd_err(g, N, ev8, col_e=1, col_q=5)
+    assert np.array_equal(b, e2) and b.sum() > 0
+    gj = _golden("binmd_hand.json")
+    grid = orc.Grid(gj["grid"]["lo"], gj["grid"]["hi"], gj["grid"]["n"])
+    hev = np.array(gj["events"], dtype=np.float32)
+    hev8 = np.zeros((len(hev), 8), np.float32)
+    hev8[:, 0] = hev[:, 0]
+    hev8[:, 1] = hev[:, 0] ** 2
+    hev8[:, 5:8] = hev[:, 1:4]
+    he = orc.binmd_err(grid, np.array(gj["N"]), hev8, col_e=1, col_q=5)
+    expect = np.zeros(grid.nbins)
+    expect[0], expect[3], expect[57] = 4.0 + 9.0 + 9.0, 1.0, 0.0625
+    np.testing.assert_array_equal(he, expect)
+    norm = orc.mdnorm(g, wl.pix_dir[::97], wl.solid[::97], wl.flux_k, wl.flux_F,
+                      orc.mdnorm_matrices(wl.R, wl.UB, wl.ops, wl.W), 1.0, wl.k_min, wl.k_max)
+    x1, s1 = orc.cross_section(b, norm), orc.cross_section_err(e2, norm)
+    x2, s2 = orc.cross_section(2 * b, 2 * norm), orc.cross_section_err(2 * e2, 2 * norm)
+    ok = ~np.isnan(x1)
+    assert np.array_equal(np.isnan(s1), np.isnan(x1))
+    np.testing.assert_allclose(x2[ok], x1[ok], rtol=1e-15)
+    np.testing.assert_allclose(s2[ok], s1[ok] / math.sqrt(2.0), rtol=1e-15)
