@@ -91,6 +91,15 @@ mdn_status mdnorm_set_pixel_krange(mdn_grid *g, int64_t npix, const double *kmin
  * F is clamped to F[0] below k[0] and to F[n-1] above k[n-1]. */
 mdn_status mdnorm_set_flux(mdn_grid *g, int64_t n, const double *k, const double *F);
 
+/* Per-bank flux tables: ntables cumulative-flux tables concatenated in
+ * k/F (host or device), table t = [offsets[t], offsets[t+1]) (offsets: int64[ntables+1], host,
+ * offsets[0] == 0, every table >= 2 knots with the rules of mdnorm_set_flux), and pixel_table:
+ * int32[npix] (host or device) giving each pixel's table (required when ntables > 1; npix must
+ * equal the instrument's).  Replaces any earlier flux; a later set_instrument drops a pixel map
+ * (the tables must then be set again).  mdnorm_set_flux(n, k, F) == one table, no map. */
+mdn_status mdnorm_set_flux_tables(mdn_grid *g, int32_t ntables, const int64_t *offsets, const double *k,
+                                  const double *F, int64_t npix, const int32_t *pixel_table);
+
 /* MDNorm of one run (Algorithm 1 line "mdnorm += MDNorm"): all nops symmetry ops
  * (ops: double[nops][9], host) x pixels p = pix_begin, pix_begin + pix_stride, ... < pix_end
  * (the shard; pix_end = -1 means npix).  UB, R: double[9] host (R = goniometer rotation of the

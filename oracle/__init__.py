@@ -65,6 +65,9 @@ def lib():
         _lib.orc_mdnorm_krange.argtypes = [P, i64, P, P, P, P, i64, P, P, i32, P, P, d, d, i64, i64, i64,
                                            P, P]
         _lib.orc_mdnorm_krange.restype = i64
+        _lib.orc_mdnorm_tables.argtypes = [P, i64, P, P, P, P, i32, P, P, P, P, i32, P, P, d, d, i64, i64,
+                                           i64, P, P]
+        _lib.orc_mdnorm_tables.restype = i64
         _lib.orc_binmd_err.argtypes = [P, i32, P, i64, P, i64, i32, i32, P, P]
         _lib.orc_binmd_err.restype = i64
         _lib.orc_cross_section_err.argtypes = [i64, P, P, P]
@@ -165,6 +168,29 @@ def mdnorm_krange(grid: Grid, pix_dir, solid, pix_kmin, pix_kmax, fk, fF, M, cha
                             None if hi is None else _p(hi), len(fk), _p(fk), _p(fF), len(M), _p(M),
                             _p(charge), float(k_min), float(k_max), int(pix_begin), int(pix_end),
                             int(pix_stride), _p(acc.sum), _p(acc.comp))
+    return acc.value()
+
+
+def mdnorm_tables(grid: Grid, pix_dir, solid, tables, pixel_table, M, charge, k_min, k_max,
+                  pix_kmin=None, pix_kmax=None, pix_begin=0, pix_end=None, pix_stride=1,
+                  acc: Accumulator | None = None) -> np.ndarray:
+    """mdnorm with per-bank flux tables: tables = [(k, F), ...], pixel_table[p] = table index."""
+    d, s = _f64(pix_dir), _f64(solid)
+    fk = _f64(np.concatenate([t[0] for t in tables]))
+    fF = _f64(np.concatenate([t[1] for t in tables]))
+    offs = np.ascontiguousarray(np.concatenate([[0], np.cumsum([len(t[0]) for t in tables])]), dtype=np.int64)
+    pt = None if pixel_table is None else np.ascontiguousarray(pixel_table, dtype=np.int32)
+    lo = None if pix_kmin is None else _f64(pix_kmin)
+    hi = None if pix_kmax is None else _f64(pix_kmax)
+    M = _f64(M).reshape(-1, 9)
+    charge = _f64(np.broadcast_to(np.asarray(charge, dtype=np.float64), (len(M),)))
+    acc = acc or Accumulator(grid.nbins)
+    pix_end = len(s) if pix_end is None else pix_end
+    lib().orc_mdnorm_tables(grid.ref, len(s), _p(d), _p(s), None if lo is None else _p(lo),
+                            None if hi is None else _p(hi), len(tables), _p(offs), _p(fk), _p(fF),
+                            None if pt is None else _p(pt), len(M), _p(M), _p(charge), float(k_min),
+                            float(k_max), int(pix_begin), int(pix_end), int(pix_stride), _p(acc.sum),
+                            _p(acc.comp))
     return acc.value()
 
 

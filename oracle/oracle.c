@@ -243,6 +243,21 @@ int64_t orc_mdnorm_krange(const orc_grid *g, int64_t npix, const double *dir, co
                           double k_min, double k_max,
                           int64_t pix_begin, int64_t pix_end, int64_t pix_stride,
                           double *norm_sum, double *norm_comp) {
+  const int64_t offsets[2] = {0, nflux};
+  return orc_mdnorm_tables(g, npix, dir, solid, pix_kmin, pix_kmax, 1, offsets, fk, fF, NULL, nmat,
+                           M, charge, k_min, k_max, pix_begin, pix_end, pix_stride, norm_sum,
+                           norm_comp);
+}
+
+/* Most general form: per-bank flux tables (S§8(f) NEXT #1).  Table t is fk/fF[offsets[t] ..
+ * offsets[t+1]); pixel p uses table pixel_table[p] (NULL: table 0 for every pixel). */
+int64_t orc_mdnorm_tables(const orc_grid *g, int64_t npix, const double *dir, const double *solid,
+                          const double *pix_kmin, const double *pix_kmax, int32_t ntables,
+                          const int64_t *offsets, const double *fk, const double *fF,
+                          const int32_t *pixel_table, int32_t nmat, const double *M,
+                          const double *charge, double k_min, double k_max, int64_t pix_begin,
+                          int64_t pix_end, int64_t pix_stride, double *norm_sum, double *norm_comp) {
+  (void)ntables;
   gconst c;
   grid_consts(g, &c);
   if (pix_end > npix) pix_end = npix;
@@ -254,7 +269,9 @@ int64_t orc_mdnorm_krange(const orc_grid *g, int64_t npix, const double *dir, co
       double lo = k_min, hi = k_max;
       if (pix_kmin && pix_kmin[p] > lo) lo = pix_kmin[p];
       if (pix_kmax && pix_kmax[p] < hi) hi = pix_kmax[p];
-      trajectory(&c, dir + 3 * p, solid[p] * charge[m], nflux, fk, fF, M + 9 * m, lo, hi, buf,
+      const int32_t t = pixel_table ? pixel_table[p] : 0;
+      const int64_t o = offsets[t], nf = offsets[t + 1] - offsets[t];
+      trajectory(&c, dir + 3 * p, solid[p] * charge[m], nf, fk + o, fF + o, M + 9 * m, lo, hi, buf,
                  &ncross, NULL, NULL, 0, norm_sum, norm_comp);
       ++ntraj;
     }

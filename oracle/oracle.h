@@ -62,6 +62,15 @@ int64_t orc_mdnorm_krange(const orc_grid *g, int64_t npix, const double *dir, co
                           int64_t pix_begin, int64_t pix_end, int64_t pix_stride,
                           double *norm_sum, double *norm_comp);
 
+/* Most general form: per-bank flux tables.  Table t = fk/fF[offsets[t] .. offsets[t+1]); pixel p
+ * uses table pixel_table[p] (NULL: table 0).  Optional per-pixel limits as above. */
+int64_t orc_mdnorm_tables(const orc_grid *g, int64_t npix, const double *dir, const double *solid,
+                          const double *pix_kmin, const double *pix_kmax, int32_t ntables,
+                          const int64_t *offsets, const double *fk, const double *fF,
+                          const int32_t *pixel_table, int32_t nmat, const double *M,
+                          const double *charge, double k_min, double k_max, int64_t pix_begin,
+                          int64_t pix_end, int64_t pix_stride, double *norm_sum, double *norm_comp);
+
 /* One trajectory, for bit-exact debug checks: n_cross = |L| (endpoints + kept crossings),
  * n_seg = number of segments appended, seg_bins/seg_vals = the first max_segs of them in order.
  * Returns n_seg. */

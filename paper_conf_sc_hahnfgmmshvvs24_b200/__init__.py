@@ -8,7 +8,7 @@ from .mdnorm import (  # noqa: F401
     mdnorm_create_grid, mdnorm_destroy, mdnorm_set_instrument, mdnorm_set_flux,
     mdnorm_accumulate, mdnorm_accumulate_runs, binmd_accumulate, mdnorm_histograms,
     mdnorm_cross_section, mdnorm_reset, mdnorm_stats, mdn_last_error, mdn_version,
-    mdnorm_set_pixel_krange, binmd_accumulate_err, mdnorm_error_histogram, mdnorm_cross_section_err,
+    mdnorm_set_pixel_krange, mdnorm_set_flux_tables, binmd_accumulate_err, mdnorm_error_histogram, mdnorm_cross_section_err,
     mdnorm_accumulate_matrices, binmd_accumulate_matrices, mdnorm_debug_trajectories,
     binmd_debug_bins, mdnorm_debug_compose, packed_histograms,
 )

@@ -34,6 +34,7 @@ SIGNATURES = {
     "mdnorm_cross_section": [P, P, P],
     "mdnorm_reset": [P, P],
     "mdnorm_set_pixel_krange": [P, i64, P, P],
+    "mdnorm_set_flux_tables": [P, i32, P, P, P, i64, P],
     "binmd_accumulate_err": [P, P, i32, P, i64, P, i64, i32, i32, i32, P],
     "mdnorm_error_histogram": [P, P],
     "mdnorm_cross_section_err": [P, P, P, P],

@@ -27,12 +27,12 @@ struct mdn_grid {
   double2* d_pkr = nullptr;  // per-pixel (k_lo, k_hi) limits, or nullptr
   double4* d_pix = nullptr;
   int64_t npix = 0;
-  double2* d_flux = nullptr;  // (kappa_i, Phi_i), nflux entries
-  int* d_ftab = nullptr;      // flux search start table (nftab cells)
-  int32_t nflux = 0, nftab = 0;
-  double ftab_k0 = 0.0, ftab_inv_cell = 0.0;
-  int ftab_nsteps = 0;
-  double flux_F_first = 0.0, flux_k_last = 0.0, flux_F_last = 0.0;
+  double2* d_flux = nullptr;  // knots of every flux table, (kappa_i, Phi_i) + 2 pads each
+  int* d_ftab = nullptr;      // cell tables of every flux table
+  mdn::FluxView* d_fviews = nullptr;  // one view per flux table (device)
+  int32_t* d_ptab = nullptr;  // pixel -> flux table (several tables only)
+  int32_t nftables = 0;
+  mdn::FluxView flux0{};      // view of table 0 (device pointers)
   mdn::Hitter* d_hit = nullptr;       // cull -> walk hand-off buffer
   uint32_t hit_cap = 0;
   mdn::DevCounters* d_ctr = nullptr;
@@ -173,16 +173,9 @@ mdn::MdnParams mdn_params(mdn_grid* g, double k_min, double k_max, int64_t pix_b
   p.pix_begin = pix_begin;
   p.pix_stride = pix_stride;
   p.nshard = nshard;
-  p.flux.kf = g->d_flux;
-  p.flux.tab = g->d_ftab;
-  p.flux.k_first = g->ftab_k0;
-  p.flux.F_first = g->flux_F_first;
-  p.flux.k_last = g->flux_k_last;
-  p.flux.F_last = g->flux_F_last;
-  p.flux.inv_cell = g->ftab_inv_cell;
-  p.flux.n = g->nflux;
-  p.flux.ntab = g->nftab;
-  p.flux.nsteps = g->ftab_nsteps;
+  p.flux = g->flux0;
+  p.fviews = g->nftables > 1 ? g->d_fviews : nullptr;
+  p.ptab = g->nftables > 1 ? g->d_ptab : nullptr;
   p.acc_f32 = g->acc == MDN_ACC_F32;
   p.kmin = k_min;
   p.kmax = k_max;
@@ -383,6 +376,8 @@ mdn_status mdnorm_destroy(mdn_grid* g) {
   cudaFree(g->d_pkr);
   cudaFree(g->d_flux);
   cudaFree(g->d_ftab);
+  cudaFree(g->d_fviews);
+  cudaFree(g->d_ptab);
   cudaFree(g->d_hit);
   cudaFree(g->d_ctr);
   cudaFree(g->d_xs);
@@ -426,74 +421,175 @@ mdn_status mdnorm_set_instrument(mdn_grid* g, int64_t npix, const double* dir, c
   cudaFree(g->d_pix);
   cudaFree(g->d_pkr);  // per-pixel limits belong to the previous instrument
   g->d_pkr = nullptr;
+  if (g->nftables > 1) {  // so does a pixel -> flux-table map: the tables must be set again
+    cudaFree(g->d_flux);
+    cudaFree(g->d_ftab);
+    cudaFree(g->d_fviews);
+    cudaFree(g->d_ptab);
+    g->d_flux = nullptr;
+    g->d_ftab = nullptr;
+    g->d_fviews = nullptr;
+    g->d_ptab = nullptr;
+    g->nftables = 0;
+  }
   g->d_pix = d_pix;
   g->npix = npix;
   return ok();
 }
 
-mdn_status mdnorm_set_flux(mdn_grid* g, int64_t n, const double* k, const double* F) {
-  if (!g) return fail(MDN_EINVAL, "grid is NULL");
-  if (n < 2 || n > (1 << 30) || !k || !F) return fail(MDN_EINVAL, "need n >= 2 and non-NULL k, F");
-  DeviceGuard dg(g->device);
-  std::vector<double> hk, hF;
-  MDN_CUDA(to_host(k, n, hk), "read k");
-  MDN_CUDA(to_host(F, n, hF), "read F");
-  if (!finite_all(hk.data(), n) || !finite_all(hF.data(), n)) return fail(MDN_EINVAL, "flux table has non-finite values");
+namespace {
+
+// Host image of one flux table (M5): knots (kappa_i, Phi_i) + two (+inf, +inf) pads, and the
+// cell table of flux_at: tab[c] = max{i : kappa_i <= fl(kappa_0 + c * cell)} (exact
+// comparisons, capped at n - 2), flagged dense when cell c holds more than three knots.
+// 4n cells for a single table staged in shared memory (uint16 copy), 2n otherwise.
+struct HostFluxTable {
+  std::vector<double2> kf;
+  std::vector<int> tab;
+  double k_first, F_first, k_last, F_last, inv_cell;
+  int n, ntab, nsteps;
+};
+
+mdn_status build_flux_table(const double* hk, const double* hF, int64_t n, bool smem_cells, HostFluxTable& t) {
+  if (n < 2 || n > (1 << 28)) return fail(MDN_EINVAL, "a flux table needs 2 .. 2^28 knots (got %lld)", (long long)n);
+  if (!finite_all(hk, n) || !finite_all(hF, n)) return fail(MDN_EINVAL, "flux table has non-finite values");
   for (int64_t i = 1; i < n; ++i) {
     if (!(hk[i] > hk[i - 1])) return fail(MDN_EINVAL, "flux k not strictly increasing at %lld", (long long)i);
     if (hF[i] < hF[i - 1]) return fail(MDN_EINVAL, "cumulative flux F decreases at %lld", (long long)i);
   }
-  // (kappa_i, Phi_i) interleaved + two (+inf, +inf) pads, plus the cell table of flux_at (M5):
-  // 4n uniform cells for tables staged in shared memory (uint16 copy), 2n otherwise
-  std::vector<double2> kf((size_t)n + 2);
-  for (int64_t i = 0; i < n; ++i) kf[i] = make_double2(hk[i], hF[i]);
-  kf[n] = kf[n + 1] = make_double2(HUGE_VAL, HUGE_VAL);
-  const int ntab = (int)std::min<int64_t>((n <= mdn::kFluxSmemMax ? 4 : 2) * n, 1 << 22);
+  t.kf.resize((size_t)n + 2);
+  for (int64_t i = 0; i < n; ++i) t.kf[i] = make_double2(hk[i], hF[i]);
+  t.kf[n] = t.kf[n + 1] = make_double2(HUGE_VAL, HUGE_VAL);
+  const int ntab = (int)std::min<int64_t>((smem_cells && n <= mdn::kFluxSmemMax ? 4 : 2) * n, 1 << 22);
   const double cell = (hk[n - 1] - hk[0]) / (double)ntab;
-  // tab[c] = max{i : kappa_i <= fl(kappa_0 + c * cell)} (exact comparisons, capped at n - 2),
-  // flagged dense when cell c holds more than three knots (tab[c+1] - tab[c] > 3)
-  std::vector<int> htab((size_t)ntab);
+  t.tab.resize((size_t)ntab);
   for (int c = 0, i = 0; c < ntab; ++c) {
     const double x = hk[0] + (double)c * cell;
     while (i + 1 < n - 1 && hk[i + 1] <= x) ++i;
-    htab[c] = i;
+    t.tab[c] = i;
   }
   int wmax = 1;
   for (int c = 0; c < ntab; ++c) {
-    const int lo = htab[std::max(c - 1, 0)];
-    const int hi = c + 2 < ntab ? htab[c + 2] + 1 : (int)n - 1;
+    const int lo = t.tab[std::max(c - 1, 0)];
+    const int hi = c + 2 < ntab ? t.tab[c + 2] + 1 : (int)n - 1;
     wmax = std::max(wmax, hi - lo);
   }
   for (int c = 0; c < ntab; ++c) {
-    const bool dense = c + 1 >= ntab || (htab[c + 1] & (int)(mdn::kFluxDense32 - 1)) - htab[c] > 3;
-    if (dense) htab[c] |= (int)mdn::kFluxDense32;
+    const bool dense = c + 1 >= ntab || (t.tab[c + 1] & (int)(mdn::kFluxDense32 - 1)) - t.tab[c] > 3;
+    if (dense) t.tab[c] |= (int)mdn::kFluxDense32;
   }
-  int nsteps = 0;
-  while ((1 << nsteps) < wmax) ++nsteps;
+  t.nsteps = 0;
+  while ((1 << t.nsteps) < wmax) ++t.nsteps;
+  t.k_first = hk[0];
+  t.F_first = hF[0];
+  t.k_last = hk[n - 1];
+  t.F_last = hF[n - 1];
+  t.inv_cell = 1.0 / cell;
+  t.n = (int)n;
+  t.ntab = ntab;
+  return MDN_OK;
+}
+
+}  // namespace
+
+mdn_status mdnorm_set_flux_tables(mdn_grid* g, int32_t ntables, const int64_t* offsets, const double* k,
+                                  const double* F, int64_t npix, const int32_t* pixel_table) {
+  if (!g) return fail(MDN_EINVAL, "grid is NULL");
+  if (ntables < 1 || ntables > (1 << 20) || !offsets || !k || !F)
+    return fail(MDN_EINVAL, "need ntables >= 1 and non-NULL offsets, k, F");
+  if (ntables > 1 && !pixel_table) return fail(MDN_EINVAL, "several flux tables need a pixel -> table map");
+  if (pixel_table && (!g->d_pix || npix != g->npix))
+    return fail(MDN_EINVAL, "the pixel -> table map needs npix == the instrument's (%lld)", (long long)g->npix);
+  if (offsets[0] != 0) return fail(MDN_EINVAL, "offsets[0] must be 0");
+  for (int t = 0; t < ntables; ++t)
+    if (offsets[t + 1] - offsets[t] < 2) return fail(MDN_EINVAL, "flux table %d has fewer than 2 knots", t);
+  const int64_t total = offsets[ntables];
+  DeviceGuard dg(g->device);
+  std::vector<double> hk, hF;
+  MDN_CUDA(to_host(k, total, hk), "read k");
+  MDN_CUDA(to_host(F, total, hF), "read F");
+  std::vector<int32_t> hpt;
+  if (pixel_table) {
+    MDN_CUDA(to_host(pixel_table, npix, hpt), "read pixel table");
+    for (int64_t i = 0; i < npix; ++i)
+      if (hpt[i] < 0 || hpt[i] >= ntables) return fail(MDN_EINVAL, "pixel_table[%lld] = %d outside [0, %d)", (long long)i, hpt[i], ntables);
+  }
+  std::vector<HostFluxTable> tabs((size_t)ntables);
+  mdn_status st;
+  for (int t = 0; t < ntables; ++t)
+    if ((st = build_flux_table(hk.data() + offsets[t], hF.data() + offsets[t], offsets[t + 1] - offsets[t],
+                               ntables == 1, tabs[t])) != MDN_OK)
+      return st;
+  // concatenate: knots and cell tables of every table, then one FluxView per table
+  size_t nkf = 0, ntb = 0;
+  for (auto& t : tabs) {
+    nkf += t.kf.size();
+    ntb += t.tab.size();
+  }
+  std::vector<double2> all_kf;
+  std::vector<int> all_tab;
+  all_kf.reserve(nkf);
+  all_tab.reserve(ntb);
+  std::vector<size_t> kf_off, tb_off;
+  for (auto& t : tabs) {
+    kf_off.push_back(all_kf.size());
+    tb_off.push_back(all_tab.size());
+    all_kf.insert(all_kf.end(), t.kf.begin(), t.kf.end());
+    all_tab.insert(all_tab.end(), t.tab.begin(), t.tab.end());
+  }
   double2* d = nullptr;
   int* tab = nullptr;
-  cudaError_t e = cudaMalloc(&d, sizeof(double2) * (n + 2));
-  if (e == cudaSuccess) e = cudaMalloc(&tab, sizeof(int) * ntab);
-  if (e == cudaSuccess) e = cudaMemcpy(d, kf.data(), sizeof(double2) * (n + 2), cudaMemcpyHostToDevice);
-  if (e == cudaSuccess) e = cudaMemcpy(tab, htab.data(), sizeof(int) * ntab, cudaMemcpyHostToDevice);
+  mdn::FluxView* views = nullptr;
+  int32_t* ptab = nullptr;
+  cudaError_t e = cudaMalloc(&d, sizeof(double2) * nkf);
+  if (e == cudaSuccess) e = cudaMalloc(&tab, sizeof(int) * ntb);
+  if (e == cudaSuccess) e = cudaMalloc(&views, sizeof(mdn::FluxView) * ntables);
+  if (e == cudaSuccess && pixel_table && ntables > 1) e = cudaMalloc(&ptab, sizeof(int32_t) * npix);
+  std::vector<mdn::FluxView> hv((size_t)ntables);
+  for (int t = 0; t < ntables; ++t) {
+    mdn::FluxView& v = hv[t];
+    v = mdn::FluxView{};
+    v.kf = d + kf_off[t];
+    v.tab = tab + tb_off[t];
+    v.k_first = tabs[t].k_first;
+    v.F_first = tabs[t].F_first;
+    v.k_last = tabs[t].k_last;
+    v.F_last = tabs[t].F_last;
+    v.inv_cell = tabs[t].inv_cell;
+    v.n = tabs[t].n;
+    v.ntab = tabs[t].ntab;
+    v.nsteps = tabs[t].nsteps;
+  }
+  if (e == cudaSuccess) e = cudaMemcpy(d, all_kf.data(), sizeof(double2) * nkf, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemcpy(tab, all_tab.data(), sizeof(int) * ntb, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemcpy(views, hv.data(), sizeof(mdn::FluxView) * ntables, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess && ptab) e = cudaMemcpy(ptab, hpt.data(), sizeof(int32_t) * npix, cudaMemcpyHostToDevice);
   if (e != cudaSuccess) {
     cudaFree(d);
     cudaFree(tab);
+    cudaFree(views);
+    cudaFree(ptab);
     return cuda_fail(e, "set_flux");
   }
+  cudaDeviceSynchronize();
   cudaFree(g->d_flux);
   cudaFree(g->d_ftab);
+  cudaFree(g->d_fviews);
+  cudaFree(g->d_ptab);
   g->d_flux = d;
   g->d_ftab = tab;
-  g->nflux = (int32_t)n;
-  g->nftab = ntab;
-  g->ftab_k0 = hk[0];
-  g->ftab_inv_cell = 1.0 / cell;
-  g->ftab_nsteps = nsteps;
-  g->flux_F_first = hF[0];
-  g->flux_k_last = hk[n - 1];
-  g->flux_F_last = hF[n - 1];
+  g->d_fviews = views;
+  g->d_ptab = ptab;
+  g->nftables = ntables;
+  g->flux0 = hv[0];
   return ok();
+}
+
+mdn_status mdnorm_set_flux(mdn_grid* g, int64_t n, const double* k, const double* F) {
+  if (!g) return fail(MDN_EINVAL, "grid is NULL");
+  if (n < 2 || !k || !F) return fail(MDN_EINVAL, "need n >= 2 and non-NULL k, F");
+  const int64_t offsets[2] = {0, n};
+  return mdnorm_set_flux_tables(g, 1, offsets, k, F, 0, nullptr);
 }
 
 mdn_status mdnorm_accumulate_runs(mdn_grid* g, const double UB[9], int32_t nruns, const double* R,

@@ -170,7 +170,8 @@ mdnorm_cull_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ 
           }
           h.v0 = v0; h.v1 = v1; h.v2 = v2; h.kin = kin; h.kout = kout;
           h.oc = dmul(px.w, sC[m]);
-          h.A = A; h.jA = sa.j; h.stepG = sa.step * G; h.P = P;
+          h.A = A | ((p.ptab ? p.ptab[pixel] : 0) << 2);  // busiest axis | flux table << 2
+          h.jA = sa.j; h.stepG = sa.step * G; h.P = P;
           if (kStats) {
             c_hit += 1;
             c_cross += total;
@@ -236,9 +237,12 @@ mdnorm_cull_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ 
 }
 
 // ---------------------------------------------------------------- M3-M7: balanced piece walk
-template <bool kSmemFlux, bool kStats, bool k3D>
+// kFlux: 0 = one flux table read from global memory, 1 = one table staged in shared memory,
+// 2 = per-bank tables (pixel -> table map, NEXT #1) read from global memory
+template <int kFlux, bool kStats, bool k3D>
 __global__ void __launch_bounds__(walk_threads(k3D), MDN_WALK_MINB)
 mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
+  constexpr bool kSmemFlux = kFlux == 1;
   extern __shared__ double2 wsm[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int nwarps = blockDim.x >> 5;
@@ -296,17 +300,24 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
         const int pi = q - (l ? pre[l - 1] : 0);
         const Hitter& h = p.hit[h0 + l];
         const double v0 = h.v0, v1 = h.v1, v2 = h.v2;
+        const int A = h.A & 3;
         double lo_k = h.kin, hi_k = h.kout;
         if (h.P > 1) {
-          const double vA = h.A == 0 ? v0 : (h.A == 1 ? v1 : v2);
+          const double vA = A == 0 ? v0 : (A == 1 ? v1 : v2);
           const double rA = ddiv(1.0, vA);
-          if (pi > 0) lo_k = plane_k(p.g, h.A, h.jA + pi * h.stepG, rA);
-          if (pi < h.P - 1) hi_k = plane_k(p.g, h.A, h.jA + (pi + 1) * h.stepG, rA);
+          if (pi > 0) lo_k = plane_k(p.g, A, h.jA + pi * h.stepG, rA);
+          if (pi < h.P - 1) hi_k = plane_k(p.g, A, h.jA + (pi + 1) * h.stepG, rA);
         }
         int nc;
-        const int ns = kSmemFlux
-                           ? traj_walk<k3D, uint16_t>(p.g, fx, v0, v1, v2, lo_k, hi_k, h.oc, emit, &nc)
-                           : traj_walk<k3D, int>(p.g, fx, v0, v1, v2, lo_k, hi_k, h.oc, emit, &nc);
+        int ns;
+        if (kFlux == 1) {
+          ns = traj_walk<k3D, uint16_t>(p.g, fx, v0, v1, v2, lo_k, hi_k, h.oc, emit, &nc);
+        } else if (kFlux == 2) {
+          const FluxView fv = p.fviews[h.A >> 2];
+          ns = traj_walk<k3D, int>(p.g, fv, v0, v1, v2, lo_k, hi_k, h.oc, emit, &nc);
+        } else {
+          ns = traj_walk<k3D, int>(p.g, fx, v0, v1, v2, lo_k, hi_k, h.oc, emit, &nc);
+        }
         if (kStats) c_seg += ns;
       }
       __syncwarp();
@@ -610,7 +621,8 @@ debug_traj_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ M
   }
   RecordEmit rec{seg_bins + t * max_segs, seg_vals + t * max_segs, max_segs, 0};
   int nc;
-  n_seg[t] = traj_walk<true>(p.g, p.flux, v[0], v[1], v[2], kin, kout, dmul(px.w, sC[m]), rec, &nc);
+  const FluxView fv = p.fviews ? p.fviews[p.ptab[pi]] : p.flux;
+  n_seg[t] = traj_walk<true>(p.g, fv, v[0], v[1], v[2], kin, kout, dmul(px.w, sC[m]), rec, &nc);
   n_cross[t] = nc + 2;  // |L| = clip endpoints + crossings
 }
 
@@ -648,12 +660,13 @@ int grid_for(int64_t work, int num_sms, int per_sm, int threads = kThreads) {
   return (int)std::max<int64_t>(blocks, 1);
 }
 
-template <bool kSmemFlux, bool kStats, bool k3D>
+template <int kFlux, bool kStats, bool k3D>
 cudaError_t launch_walk(const MdnParams& p, int num_sms, cudaStream_t s) {
+  constexpr bool kSmemFlux = kFlux == 1;
   constexpr int threads = walk_threads(k3D);
   const size_t smem = (kSmemFlux ? sizeof(double2) * (p.flux.n + 2) + sizeof(uint16_t) * ((p.flux.ntab + 1) & ~1) : 0) +
                       sizeof(int) * 32 * (threads / 32);
-  auto k = mdnorm_walk_kernel<kSmemFlux, kStats, k3D>;
+  auto k = mdnorm_walk_kernel<kFlux, kStats, k3D>;
   cudaError_t err = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (err != cudaSuccess) return err;
   int per_sm = 0;
@@ -709,13 +722,15 @@ cudaError_t launch_mdnorm(const MdnParams& p, const MatBlock& mb, int num_sms, c
   err = p.stats ? launch_cull<true>(p, mb, num_sms, s) : launch_cull<false>(p, mb, num_sms, s);
   if (err != cudaSuccess) return err;
   // 2-D slices (a single bin on the last axis, "lBins=1") merge two crossing streams
-  const bool smem_flux = p.flux.n <= kFluxSmemMax, d3 = p.g.n[2] > 1;
-  if (smem_flux) {
-    if (d3) return p.stats ? launch_walk<true, true, true>(p, num_sms, s) : launch_walk<true, false, true>(p, num_sms, s);
-    return p.stats ? launch_walk<true, true, false>(p, num_sms, s) : launch_walk<true, false, false>(p, num_sms, s);
-  }
-  if (d3) return p.stats ? launch_walk<false, true, true>(p, num_sms, s) : launch_walk<false, false, true>(p, num_sms, s);
-  return p.stats ? launch_walk<false, true, false>(p, num_sms, s) : launch_walk<false, false, false>(p, num_sms, s);
+  const bool d3 = p.g.n[2] > 1;
+  const int mode = p.fviews ? 2 : (p.flux.n <= kFluxSmemMax ? 1 : 0);
+#define MDN_WALK_DISPATCH(F)                                                                    \
+  if (d3) return p.stats ? launch_walk<F, true, true>(p, num_sms, s) : launch_walk<F, false, true>(p, num_sms, s); \
+  return p.stats ? launch_walk<F, true, false>(p, num_sms, s) : launch_walk<F, false, false>(p, num_sms, s);
+  if (mode == 1) { MDN_WALK_DISPATCH(1) }
+  if (mode == 2) { MDN_WALK_DISPATCH(2) }
+  MDN_WALK_DISPATCH(0)
+#undef MDN_WALK_DISPATCH
 }
 
 cudaError_t launch_binmd(const BinParams& p, const MatBlock& mb, int num_sms, cudaStream_t s) {

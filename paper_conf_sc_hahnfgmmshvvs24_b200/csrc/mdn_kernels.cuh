@@ -42,7 +42,8 @@ struct MatBlock {
 struct alignas(16) Hitter {
   double v0, v1, v2, kin;
   double kout, oc;
-  int32_t A, jA, stepG, P;
+  int32_t A;               // busiest axis (bits 0-1) | flux table index << 2
+  int32_t jA, stepG, P;
 };
 
 struct DevCounters {
@@ -56,7 +57,9 @@ struct MdnParams {
   const double4* pix;      // (q0, q1, q2, Omega) per pixel, q = z - d  (M1)
   const double2* pkr;      // per-pixel (k_lo, k_hi) limits, or nullptr (NEXT #1)
   int64_t pix_begin, pix_stride, nshard;
-  FluxView flux;           // device pointers (global)
+  FluxView flux;           // table 0 (device pointers, global)
+  const FluxView* fviews;  // per-bank tables (several tables), or nullptr
+  const int32_t* ptab;     // pixel -> flux table (with fviews), or nullptr
   int32_t acc_f32;
   double kmin, kmax;
   double* norm;            // fp64 histogram (nbins)

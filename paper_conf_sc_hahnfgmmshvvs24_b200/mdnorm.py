@@ -168,6 +168,17 @@ def binmd_accumulate_err(g: Grid, UB, ops, events, stride_floats=None, col_w=0, 
                                       _stream(stream, g.device)), "binmd_accumulate_err")
 
 
+def mdnorm_set_flux_tables(g: Grid, tables, pixel_table=None) -> None:
+    """Per-bank flux tables: tables = [(k, F), ...]; pixel_table[p] = table index of pixel p."""
+    k = np.ascontiguousarray(np.concatenate([np.asarray(t[0], dtype=np.float64) for t in tables]))
+    F = np.ascontiguousarray(np.concatenate([np.asarray(t[1], dtype=np.float64) for t in tables]))
+    offs = np.ascontiguousarray(np.concatenate([[0], np.cumsum([len(t[0]) for t in tables])]), dtype=np.int64)
+    pt_p, pt_k = _arg(pixel_table, np.int32) if pixel_table is not None else (None, None)
+    npix = 0 if pixel_table is None else len(pixel_table)
+    check(load().mdnorm_set_flux_tables(g.handle, len(tables), offs.ctypes.data, k.ctypes.data, F.ctypes.data,
+                                        npix, pt_p), "mdnorm_set_flux_tables")
+
+
 def mdnorm_set_pixel_krange(g: Grid, kmin, kmax) -> None:
     """Per-pixel momentum limits (None, None removes them)."""
     if kmin is None and kmax is None:

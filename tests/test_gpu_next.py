@@ -72,6 +72,47 @@ def test_pixel_krange_parity(mdn):
         mdn.mdnorm_set_pixel_krange(g, lo[:10], hi[:10])
 
 
+@pytest.mark.parametrize("cfg", ["corelli", "topaz"])
+def test_per_bank_flux_tables(mdn, cfg):
+    """Pixel -> flux-table map: each bank (TOPAZ: 25 banks of 65536 pixels; CORELLI: 3 random
+    groups) reads its own cumulative-flux table with its own knots."""
+    wl = synth.make_workload(cfg, nops=8) if cfg == "topaz" else synth.make_workload(cfg)
+    rng = np.random.default_rng(33)
+    nt = 25 if cfg == "topaz" else 3
+    tables = []
+    for t in range(nt):
+        kk = np.sort(np.unique(np.concatenate([wl.flux_k[:: 2 + t % 3], rng.uniform(wl.flux_k[0], wl.flux_k[-1], 50)])))
+        FF = np.interp(kk, wl.flux_k, wl.flux_F) * (0.5 + rng.uniform())
+        FF[0] = 0.0
+        FF = np.maximum.accumulate(FF)
+        tables.append((kk, FF))
+    pt = (np.arange(wl.npix) // 65536).astype(np.int32) if cfg == "topaz" else \
+        rng.integers(0, nt, wl.npix).astype(np.int32)
+    g = mdn.mdnorm_create_grid(0, wl.lo, wl.hi, wl.nbins, wl.W)
+    mdn.mdnorm_set_instrument(g, wl.pix_dir, wl.solid)
+    mdn.mdnorm_set_flux_tables(g, tables, pt)
+    stride = 7 if cfg == "corelli" else 997
+    mdn.mdnorm_accumulate(g, wl.UB, wl.R[0], wl.ops, wl.k_min, wl.k_max, 1.0, pix_stride=stride)
+    norm, _, _ = _packed(mdn, g)
+    og = oracle.workload_grid(wl)
+    M = oracle.mdnorm_matrices(wl.R, wl.UB, wl.ops, wl.W)
+    onorm = oracle.mdnorm_tables(og, wl.pix_dir, wl.solid, tables, pt, M, 1.0, wl.k_min, wl.k_max,
+                                 pix_stride=stride)
+    assert onorm.sum() > 0
+    _assert_rel(norm, onorm)
+    ids = rng.integers(0, len(M) * wl.npix, size=1500)
+    nc, ns, bins, vals = mdn.mdnorm_debug_trajectories(g, M, np.ones(len(M)), wl.k_min, wl.k_max, ids, 700)
+    for t, tid in enumerate(ids):
+        m, p = divmod(int(tid), wl.npix)
+        kk, FF = tables[pt[p]]
+        onc, ons, ob, ov = oracle.mdnorm_trajectory(og, wl.pix_dir[p], wl.solid[p], kk, FF, M[m], 1.0,
+                                                    wl.k_min, wl.k_max, 700)
+        assert (nc[t], ns[t]) == (onc, ons)
+        assert np.array_equal(bins[t, :ons], ob) and np.array_equal(vals[t, :ons], ov)
+    with pytest.raises(mdn.MdnError, match="MDN_EINVAL"):
+        mdn.mdnorm_set_flux_tables(g, tables, np.full(wl.npix, nt, np.int32))
+
+
 def test_error_histogram_and_xs_err(mdn):
     import torch
     wl = synth.make_workload("corelli", events_per_run=1_000_000)
