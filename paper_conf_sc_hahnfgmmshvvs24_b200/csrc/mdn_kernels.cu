@@ -58,6 +58,19 @@ __device__ __forceinline__ void stage_binmd_mats(const MatBlock& mb, double* sN)
   }
 }
 
+// Warp min / max of a float with one REDUX each: IEEE floats compare like the signed integers
+// i ^ ((i >> 31) & 0x7fffffff) (an involution), and __reduce_{min,max}_sync reduce ints.
+__device__ __forceinline__ int float_key(float f) {
+  const int i = __float_as_int(f);
+  return i ^ ((i >> 31) & 0x7fffffff);
+}
+__device__ __forceinline__ float warp_min(float f) {
+  return __int_as_float(float_key(__int_as_float(__reduce_min_sync(0xffffffffu, float_key(f)))));
+}
+__device__ __forceinline__ float warp_max(float f) {
+  return __int_as_float(float_key(__int_as_float(__reduce_max_sync(0xffffffffu, float_key(f)))));
+}
+
 // One warp-aggregated atomic per counter per warp (tracing only; compiled out when kStats off).
 __device__ __forceinline__ void flush_counter(unsigned long long* dst, unsigned long long v) {
 #pragma unroll
@@ -502,9 +515,31 @@ binmd_kernel(const __grid_constant__ BinParams p, const __grid_constant__ MatBlo
     const float q0 = cur.y, q1 = cur.z, q2 = cur.w;
     const float qm = fmaxf(fabsf(q0), fmaxf(fabsf(q1), fabsf(q2)));
     if (kStats && valid) c_pairs += mb.nmat;
+#ifdef MDN_BINMD_BOX
+    // Warp box (S§8(f) NEXT #4, Mantid's MDBox idea on the Morton-ordered stream): the 32
+    // events' Q bounding box, transformed by interval arithmetic, rejects a whole class at once
+    // when it misses [0, n) on the class axis by more than the fp32 error bound.  Measured
+    // slower than the per-event test on the CORELLI slab, so it is off.
+    const float b0l = warp_min(valid ? q0 : CUDART_INF_F), b0h = warp_max(valid ? q0 : -CUDART_INF_F);
+    const float b1l = warp_min(valid ? q1 : CUDART_INF_F), b1h = warp_max(valid ? q1 : -CUDART_INF_F);
+    const float b2l = warp_min(valid ? q2 : CUDART_INF_F), b2h = warp_max(valid ? q2 : -CUDART_INF_F);
+    const float bqm = fmaxf(fmaxf(fmaxf(fabsf(b0l), fabsf(b0h)), fmaxf(fabsf(b1l), fabsf(b1h))),
+                            fmaxf(fabsf(b2l), fabsf(b2h)));
+#endif
     for (int c = 0; c < ncls; ++c) {
       // first-tested axis, once for the whole class
       const BinAxis32 ax = sA[3 * sMem[sCls[c]]];
+#ifdef MDN_BINMD_BOX
+      {  // warp-uniform box test
+        const float p0a = ax.r0 * b0l, p0b = ax.r0 * b0h, p1a = ax.r1 * b1l, p1b = ax.r1 * b1h;
+        const float p2a = ax.r2 * b2l, p2b = ax.r2 * b2h;
+        const float xl = fminf(p0a, p0b) + fminf(p1a, p1b) + fminf(p2a, p2b);
+        const float xh = fmaxf(p0a, p0b) + fmaxf(p1a, p1b) + fmaxf(p2a, p2b);
+        const float tl = fmaf(xl, ax.s, -ax.los), th = fmaf(xh, ax.s, -ax.los);
+        const float bdl = 2.0f * fmaf(ax.c, bqm, ax.d);
+        if (th < -bdl || tl >= ax.n + bdl) continue;  // no event of this warp can land: skip
+      }
+#endif
       const float x = fmaf(ax.r2, q2, fmaf(ax.r1, q1, ax.r0 * q0));
       const float t = fmaf(x, ax.s, -ax.los);
       const float dl = fmaf(ax.c, qm, ax.d);
