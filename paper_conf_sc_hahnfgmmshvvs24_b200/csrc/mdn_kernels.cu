@@ -58,6 +58,7 @@ __device__ __forceinline__ void stage_binmd_mats(const MatBlock& mb, double* sN)
   }
 }
 
+#ifdef MDN_BINMD_BOX
 // Warp min / max of a float with one REDUX each: IEEE floats compare like the signed integers
 // i ^ ((i >> 31) & 0x7fffffff) (an involution), and __reduce_{min,max}_sync reduce ints.
 __device__ __forceinline__ int float_key(float f) {
@@ -70,6 +71,7 @@ __device__ __forceinline__ float warp_min(float f) {
 __device__ __forceinline__ float warp_max(float f) {
   return __int_as_float(float_key(__int_as_float(__reduce_max_sync(0xffffffffu, float_key(f)))));
 }
+#endif
 
 // One warp-aggregated atomic per counter per warp (tracing only; compiled out when kStats off).
 __device__ __forceinline__ void flush_counter(unsigned long long* dst, unsigned long long v) {
