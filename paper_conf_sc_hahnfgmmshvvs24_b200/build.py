@@ -17,6 +17,8 @@ NVCC_FLAGS = [
     # geometry must be bit-identical to the fp64 definition: no mul+add contraction anywhere
     # (the code also uses explicit __dmul_rn/__dadd_rn intrinsics; this is the guard)
     "--fmad=false",
+    # host side: the flux cell table evaluates the device's U(x) expression (mdn_api.cu)
+    "-Xcompiler", "-ffp-contract=off",
     "-Xcompiler", "-fPIC", "-Xcompiler", "-Wall", "-shared", "-cudart", "static",
 ]
 

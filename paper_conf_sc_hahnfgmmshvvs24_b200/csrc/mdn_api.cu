@@ -27,7 +27,7 @@ struct mdn_grid {
   double2* d_pkr = nullptr;  // per-pixel (k_lo, k_hi) limits, or nullptr
   double4* d_pix = nullptr;
   int64_t npix = 0;
-  double2* d_flux = nullptr;  // knots of every flux table, (kappa_i, Phi_i) + 2 pads each
+  double* d_flux = nullptr;   // every flux table: knots (+2 pads each), then interval records
   int* d_ftab = nullptr;      // cell tables of every flux table
   mdn::FluxView* d_fviews = nullptr;  // one view per flux table (device)
   int32_t* d_ptab = nullptr;  // pixel -> flux table (several tables only)
@@ -439,52 +439,61 @@ mdn_status mdnorm_set_instrument(mdn_grid* g, int64_t npix, const double* dir, c
 
 namespace {
 
-// Host image of one flux table (M5): knots (kappa_i, Phi_i) + two (+inf, +inf) pads, and the
-// cell table of flux_at: tab[c] = max{i : kappa_i <= fl(kappa_0 + c * cell)} (exact
-// comparisons, capped at n - 2), flagged dense when cell c holds more than three knots.
-// 4n cells for a single table staged in shared memory (uint16 copy), 2n otherwise.
+// Host image of one flux table (M5, see flux_at in mdn_device.cuh): knots kappa_i + two +inf
+// pads; per interval (Phi_i, dPhi_i, y_i, dk_i) with dPhi_i = Phi_{i+1} - Phi_i, dk_i =
+// kappa_{i+1} - kappa_i, y_i = 1 / dk_i (IEEE double, the same roundings as the device); and the
+// cell table over U(x) = (x - kappa_0) * inv_cell: entry c = s_c = max{i : U_i < c}, flagged
+// when cell c holds more than three knots, when s_c does not exist (c = 0) or when c + 1 > U_{n-1}.
+// max(2n, range / (2.9 min spacing)) cells, at most 2^22.  This file is compiled with -ffp-contract=off, so U_i is exactly the
+// device's dmul(dsub(x, kappa_0), inv_cell).
 struct HostFluxTable {
-  std::vector<double2> kf;
+  std::vector<double> kn;
+  std::vector<double4> seg;
   std::vector<int> tab;
   double k_first, F_first, k_last, F_last, inv_cell;
-  int n, ntab, nsteps;
+  int n, ntab;
 };
 
-mdn_status build_flux_table(const double* hk, const double* hF, int64_t n, bool smem_cells, HostFluxTable& t) {
+mdn_status build_flux_table(const double* hk, const double* hF, int64_t n, HostFluxTable& t) {
   if (n < 2 || n > (1 << 28)) return fail(MDN_EINVAL, "a flux table needs 2 .. 2^28 knots (got %lld)", (long long)n);
   if (!finite_all(hk, n) || !finite_all(hF, n)) return fail(MDN_EINVAL, "flux table has non-finite values");
   for (int64_t i = 1; i < n; ++i) {
     if (!(hk[i] > hk[i - 1])) return fail(MDN_EINVAL, "flux k not strictly increasing at %lld", (long long)i);
     if (hF[i] < hF[i - 1]) return fail(MDN_EINVAL, "cumulative flux F decreases at %lld", (long long)i);
   }
-  t.kf.resize((size_t)n + 2);
-  for (int64_t i = 0; i < n; ++i) t.kf[i] = make_double2(hk[i], hF[i]);
-  t.kf[n] = t.kf[n + 1] = make_double2(HUGE_VAL, HUGE_VAL);
-  const int ntab = (int)std::min<int64_t>((smem_cells && n <= mdn::kFluxSmemMax ? 4 : 2) * n, 1 << 22);
-  const double cell = (hk[n - 1] - hk[0]) / (double)ntab;
-  t.tab.resize((size_t)ntab);
-  for (int c = 0, i = 0; c < ntab; ++c) {
-    const double x = hk[0] + (double)c * cell;
-    while (i + 1 < n - 1 && hk[i + 1] <= x) ++i;
-    t.tab[c] = i;
+  t.kn.assign(hk, hk + n);
+  t.kn.push_back(HUGE_VAL);
+  t.kn.push_back(HUGE_VAL);
+  t.seg.assign((size_t)n, make_double4(0.0, 0.0, 0.0, 0.0));
+  for (int64_t i = 0; i + 1 < n; ++i) {
+    const double dk = hk[i + 1] - hk[i];
+    const double dF = hF[i + 1] - hF[i];
+    if (!std::isfinite(dk) || !std::isfinite(dF) || !std::isfinite(1.0 / dk))
+      return fail(MDN_EINVAL, "flux table interval %lld overflows", (long long)i);
+    t.seg[i] = make_double4(hF[i], dF, 1.0 / dk, dk);
   }
-  int wmax = 1;
+  // cells narrower than 3 x the smallest knot spacing hold at most 3 knots (all fast)
+  double hmin = HUGE_VAL;
+  for (int64_t i = 0; i + 1 < n; ++i) hmin = std::min(hmin, hk[i + 1] - hk[i]);
+  const double want = std::ceil((hk[n - 1] - hk[0]) / (2.9 * hmin));
+  const int ntab = (int)std::min<double>(std::max<double>(2.0 * (double)n, want), (double)(1 << 22));
+  t.inv_cell = (double)ntab / (hk[n - 1] - hk[0]);
+  if (!std::isfinite(t.inv_cell)) return fail(MDN_EINVAL, "flux table k range too small");
+  std::vector<double> U((size_t)n);
+  for (int64_t i = 0; i < n; ++i) U[i] = (hk[i] - hk[0]) * t.inv_cell;
+  t.tab.assign((size_t)ntab, 0);
+  int64_t s = -1, j = 0;  // s = max{i : U_i < c}; j = first i with U_i >= c
   for (int c = 0; c < ntab; ++c) {
-    const int lo = t.tab[std::max(c - 1, 0)];
-    const int hi = c + 2 < ntab ? t.tab[c + 2] + 1 : (int)n - 1;
-    wmax = std::max(wmax, hi - lo);
+    while (j < n && U[j] < (double)c) s = j++;
+    int64_t cnt = 0;
+    while (j + cnt < n && U[j + cnt] < (double)c + 1.0) ++cnt;
+    const bool fast = s >= 0 && cnt <= 3 && (double)c + 1.0 <= U[n - 1];
+    t.tab[c] = (int)std::max<int64_t>(s, 0) | (fast ? 0 : (int)mdn::kFluxDense32);
   }
-  for (int c = 0; c < ntab; ++c) {
-    const bool dense = c + 1 >= ntab || (t.tab[c + 1] & (int)(mdn::kFluxDense32 - 1)) - t.tab[c] > 3;
-    if (dense) t.tab[c] |= (int)mdn::kFluxDense32;
-  }
-  t.nsteps = 0;
-  while ((1 << t.nsteps) < wmax) ++t.nsteps;
   t.k_first = hk[0];
   t.F_first = hF[0];
   t.k_last = hk[n - 1];
   t.F_last = hF[n - 1];
-  t.inv_cell = 1.0 / cell;
   t.n = (int)n;
   t.ntab = ntab;
   return MDN_OK;
@@ -518,30 +527,37 @@ mdn_status mdnorm_set_flux_tables(mdn_grid* g, int32_t ntables, const int64_t* o
   mdn_status st;
   for (int t = 0; t < ntables; ++t)
     if ((st = build_flux_table(hk.data() + offsets[t], hF.data() + offsets[t], offsets[t + 1] - offsets[t],
-                               ntables == 1, tabs[t])) != MDN_OK)
+                               tabs[t])) != MDN_OK)
       return st;
-  // concatenate: knots and cell tables of every table, then one FluxView per table
-  size_t nkf = 0, ntb = 0;
+  // concatenate into one allocation: every table's knots (padded to an even count, so the
+  // interval records stay 16-byte aligned), then every table's interval records; the cell
+  // tables in a second allocation; one FluxView per table
+  size_t nkn = 0, nseg = 0, ntb = 0;
   for (auto& t : tabs) {
-    nkf += t.kf.size();
+    nkn += (t.kn.size() + 1) & ~size_t(1);
+    nseg += t.seg.size();
     ntb += t.tab.size();
   }
-  std::vector<double2> all_kf;
+  std::vector<double> all(nkn + 4 * nseg, 0.0);
   std::vector<int> all_tab;
-  all_kf.reserve(nkf);
   all_tab.reserve(ntb);
-  std::vector<size_t> kf_off, tb_off;
+  std::vector<size_t> kn_off, seg_off, tb_off;
+  size_t o = 0, so = nkn;
   for (auto& t : tabs) {
-    kf_off.push_back(all_kf.size());
+    kn_off.push_back(o);
+    seg_off.push_back(so);
     tb_off.push_back(all_tab.size());
-    all_kf.insert(all_kf.end(), t.kf.begin(), t.kf.end());
+    std::copy(t.kn.begin(), t.kn.end(), all.begin() + o);
+    std::memcpy(all.data() + so, t.seg.data(), sizeof(double4) * t.seg.size());
+    o += (t.kn.size() + 1) & ~size_t(1);
+    so += 4 * t.seg.size();
     all_tab.insert(all_tab.end(), t.tab.begin(), t.tab.end());
   }
-  double2* d = nullptr;
+  double* d = nullptr;
   int* tab = nullptr;
   mdn::FluxView* views = nullptr;
   int32_t* ptab = nullptr;
-  cudaError_t e = cudaMalloc(&d, sizeof(double2) * nkf);
+  cudaError_t e = cudaMalloc(&d, sizeof(double) * all.size());
   if (e == cudaSuccess) e = cudaMalloc(&tab, sizeof(int) * ntb);
   if (e == cudaSuccess) e = cudaMalloc(&views, sizeof(mdn::FluxView) * ntables);
   if (e == cudaSuccess && pixel_table && ntables > 1) e = cudaMalloc(&ptab, sizeof(int32_t) * npix);
@@ -549,7 +565,8 @@ mdn_status mdnorm_set_flux_tables(mdn_grid* g, int32_t ntables, const int64_t* o
   for (int t = 0; t < ntables; ++t) {
     mdn::FluxView& v = hv[t];
     v = mdn::FluxView{};
-    v.kf = d + kf_off[t];
+    v.kn = d + kn_off[t];
+    v.seg = reinterpret_cast<const double4*>(d + seg_off[t]);
     v.tab = tab + tb_off[t];
     v.k_first = tabs[t].k_first;
     v.F_first = tabs[t].F_first;
@@ -558,9 +575,8 @@ mdn_status mdnorm_set_flux_tables(mdn_grid* g, int32_t ntables, const int64_t* o
     v.inv_cell = tabs[t].inv_cell;
     v.n = tabs[t].n;
     v.ntab = tabs[t].ntab;
-    v.nsteps = tabs[t].nsteps;
   }
-  if (e == cudaSuccess) e = cudaMemcpy(d, all_kf.data(), sizeof(double2) * nkf, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemcpy(d, all.data(), sizeof(double) * all.size(), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(tab, all_tab.data(), sizeof(int) * ntb, cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(views, hv.data(), sizeof(mdn::FluxView) * ntables, cudaMemcpyHostToDevice);
   if (e == cudaSuccess && ptab) e = cudaMemcpy(ptab, hpt.data(), sizeof(int32_t) * npix, cudaMemcpyHostToDevice);

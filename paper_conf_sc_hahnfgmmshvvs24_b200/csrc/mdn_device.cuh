@@ -99,23 +99,32 @@ __device__ __forceinline__ bool compose_binmd(const double* UB, const double* S,
 // ------------------------------------------------------------------------------ M5 flux
 // F(x): clamp outside, else i = max{i : kappa_i <= x} and
 //   Phi_i + (Phi_{i+1} - Phi_i) * ((x - kappa_i) / (kappa_{i+1} - kappa_i)).
-// i is unique, so it may be found by any search.  A uniform-cell table gives
-// tab[c] = max{i : kappa_i <= fl(kappa_0 + c * cell)} (host, exact comparisons), with flag bit
-// kFluxDense set when cell c holds more than 3 knots.  The cell of x is computed from an
-// approximate u (relative error ~1e-16, i.e. ~1e-12 cells); unless u is within 1e-9 of a cell
-// boundary it is exact, so for a non-dense interior cell i is tab[c] + (#probes of the next three
-// knots that are <= x) -- independent loads, no bisection, no clamps (kappa_0 < x < kappa_{n-1}
-// there).  Everything else (cell edges, dense cells, x outside the table) takes the general
-// path: the window [tab[c-1], tab[c+2] + 1] and a scan.  The knot array is padded with two
-// (+inf, +inf) entries so the probes never read out of bounds.
+//
+// Per interval the table stores (Phi_i, dPhi_i, y_i, dk_i) with dPhi_i = RN(Phi_{i+1} - Phi_i),
+// dk_i = RN(kappa_{i+1} - kappa_i) (the same roundings as the formula) and y_i = RN(1 / dk_i).
+// The correctly rounded quotient a / dk_i (a = RN(x - kappa_i)) is then
+//   q = RN(a y_i);  r = a - q dk_i (exact, one FMA);  q' = RN(q + r y_i)   (one FMA)
+// -- Markstein's theorem: y within half an ulp of 1/b and q within one ulp of a/b make r exact
+// and q' = RN(a/b) (no overflow / underflow here: 0 <= a < dk, both normal or zero).  Three
+// fp64 instructions instead of an IEEE division; tests/test_flux_division.py pins the claim on
+// 2e7 random and adversarial operands against IEEE division.
+//
+// Search: U(x) = RN(RN(x - kappa_0) * inv_cell) is monotone non-decreasing in x, and the host
+// evaluates the same expression U_i = U(kappa_i).  For x with floor(U(x)) = c:
+//   every knot with U_i < c is < x, and every knot with U_i >= c + 1 is > x,
+// so i = s_c + #{probes kappa_{s_c+1..s_c+3} <= x} with s_c = max{i : U_i < c}, provided cell
+// c holds at most three knots (#{i : floor(U_i) = c} <= 3) and c + 1 <= U_{n-1} (then x <
+// kappa_{n-1}, no clamp).  Cells failing that (and c = 0, x outside the table) are flagged and
+// take the general path: clamps and a bisection.  Two (+inf) pad knots keep the probes in bounds.
 constexpr unsigned kFluxDense32 = 1u << 30;  // flag bit in an int32 table entry
 constexpr unsigned kFluxDense16 = 1u << 15;  // flag bit in a uint16 (shared-memory) entry
 
 struct FluxView {
-  const double2* kf;  // (kappa_i, Phi_i), n entries + 2 padding entries
-  const void* tab;    // ntab entries: int32 (global) or uint16 (shared-memory copy)
+  const double* kn;    // kappa_i: n knots + 2 (+inf) pads
+  const double4* seg;  // per interval i < n - 1: (Phi_i, dPhi_i, y_i, dk_i); n entries
+  const void* tab;     // ntab cell entries: int32 (global) or uint16 (shared-memory copy)
   double k_first, F_first, k_last, F_last, inv_cell;
-  int n, ntab, nsteps, pad;
+  int n, ntab;
 };
 
 template <typename TabT>
@@ -123,19 +132,27 @@ __device__ __forceinline__ unsigned tab_entry(const FluxView& f, int c) {
   return (unsigned)static_cast<const TabT*>(f.tab)[c];
 }
 
-template <typename TabT>
+// Phi_i + dPhi_i * RN((x - kappa_i) / dk_i) for kappa_i <= x < kappa_{i+1}
+__device__ __forceinline__ double flux_interp(const FluxView& f, int i, double x) {
+  const double4 s = f.seg[i];
+  const double a = dsub(x, f.kn[i]);
+  const double q = dmul(a, s.z);
+  const double r = __fma_rn(-q, s.w, a);
+  const double t = __fma_rn(r, s.z, q);
+  return dadd(s.x, dmul(s.y, t));
+}
+
 __device__ __forceinline__ double flux_general(const FluxView& f, double x) {
-  constexpr unsigned flag = sizeof(TabT) == 2 ? kFluxDense16 : kFluxDense32;
   if (x <= f.k_first) return f.F_first;
   if (x >= f.k_last) return f.F_last;
-  const double u = fmin(fmax((x - f.k_first) * f.inv_cell, 0.0), (double)(f.ntab - 1));
-  const int c = (int)u;  // within one cell of the true cell
-  const int lo = (int)(tab_entry<TabT>(f, max(c - 1, 0)) & (flag - 1));
-  const int hi = c + 2 < f.ntab ? (int)(tab_entry<TabT>(f, c + 2) & (flag - 1)) + 1 : f.n - 1;
-  int i = lo;  // kappa_lo <= x < kappa_hi
-  while (i + 1 < hi && f.kf[i + 1].x <= x) ++i;
-  const double2 a = f.kf[i], b = f.kf[i + 1];
-  return dadd(a.y, dmul(dsub(b.y, a.y), ddiv(dsub(x, a.x), dsub(b.x, a.x))));
+  // largest i in [0, n - 2] with kappa_i <= x (kappa_0 < x < kappa_{n-1})
+  int lo = 0, len = f.n - 1;
+  while (len > 1) {
+    const int half = len >> 1;
+    if (f.kn[lo + half] <= x) lo += half;
+    len -= half;
+  }
+  return flux_interp(f, lo, x);
 }
 
 template <typename TabT = int>
@@ -144,16 +161,11 @@ __device__ __forceinline__ double flux_at(const FluxView& f, double x) {
   return x;
 #endif
   constexpr unsigned flag = sizeof(TabT) == 2 ? kFluxDense16 : kFluxDense32;
-  const double u = (x - f.k_first) * f.inv_cell;
-  const double uf = floor(u);
-  const double fr = u - uf;
-  const bool interior = uf >= 0.0 && uf < (double)(f.ntab - 1) && fr > 1e-9 && fr < 1.0 - 1e-9;
-  const unsigned e = interior ? tab_entry<TabT>(f, (int)uf) : flag;
-  if (e & flag) return flux_general<TabT>(f, x);
-  const int i = (int)e + (f.kf[e + 1].x <= x ? 1 : 0) + (f.kf[e + 2].x <= x ? 1 : 0) +
-                (f.kf[e + 3].x <= x ? 1 : 0);
-  const double2 a = f.kf[i], b = f.kf[i + 1];
-  return dadd(a.y, dmul(dsub(b.y, a.y), ddiv(dsub(x, a.x), dsub(b.x, a.x))));
+  const int c = __double2int_rd(dmul(dsub(x, f.k_first), f.inv_cell));
+  const unsigned e = (unsigned)c < (unsigned)f.ntab ? tab_entry<TabT>(f, c) : flag;
+  if (e & flag) return flux_general(f, x);
+  const int i = (int)e + (f.kn[e + 1] <= x ? 1 : 0) + (f.kn[e + 2] <= x ? 1 : 0) + (f.kn[e + 3] <= x ? 1 : 0);
+  return flux_interp(f, i, x);
 }
 
 // ------------------------------------------------------------------------------ M1-M2

@@ -20,14 +20,17 @@ namespace mdn {
 
 namespace {
 
+// One persistent walk CTA per SM (the shared-memory flux table takes up to 180 KB): 896 threads
+// for 2-D slices (measured: 2 x 448 > 2 x 384 ~ 2 x 512 on the CORELLI slab), 768 for 3-D grids
+// (the unrolled walk needs more registers).
 #ifndef MDN_WALK_THREADS
-#define MDN_WALK_THREADS 448    // 2-D slices (measured: 448 > 384 ~ 512 on the CORELLI slab)
+#define MDN_WALK_THREADS 896
 #endif
 #ifndef MDN_WALK_THREADS_3D
-#define MDN_WALK_THREADS_3D 384  // 3-D grids (the unrolled walk needs more registers)
+#define MDN_WALK_THREADS_3D 768
 #endif
 #ifndef MDN_WALK_MINB
-#define MDN_WALK_MINB 2
+#define MDN_WALK_MINB 1
 #endif
 constexpr int kThreads = 256;
 constexpr int walk_threads(bool k3D) { return k3D ? MDN_WALK_THREADS_3D : MDN_WALK_THREADS; }
@@ -258,15 +261,19 @@ template <int kFlux, bool kStats, bool k3D>
 __global__ void __launch_bounds__(walk_threads(k3D), MDN_WALK_MINB)
 mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
   constexpr bool kSmemFlux = kFlux == 1;
-  extern __shared__ double2 wsm[];
+  extern __shared__ double4 wsm[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int nwarps = blockDim.x >> 5;
-  // shared layout: knots (n + 2 padded double2) | cell table (uint16) | per-warp prefix sums
-  double2* sKF = wsm;
-  uint16_t* sTab = reinterpret_cast<uint16_t*>(sKF + (kSmemFlux ? p.flux.n + 2 : 0));
+  // shared layout: interval records (n double4) | knots (n + 2, even) | cell table (uint16, even)
+  // | per-warp prefix sums
+  const int n_kn = kSmemFlux ? (p.flux.n + 3) & ~1 : 0;
+  double4* sSeg = wsm;
+  double* sKn = reinterpret_cast<double*>(sSeg + (kSmemFlux ? p.flux.n : 0));
+  uint16_t* sTab = reinterpret_cast<uint16_t*>(sKn + n_kn);
   int* sPre = reinterpret_cast<int*>(sTab + (kSmemFlux ? (p.flux.ntab + 1) & ~1 : 0));
   if (kSmemFlux) {
-    for (int i = threadIdx.x; i < p.flux.n + 2; i += blockDim.x) sKF[i] = p.flux.kf[i];
+    for (int i = threadIdx.x; i < p.flux.n; i += blockDim.x) sSeg[i] = p.flux.seg[i];
+    for (int i = threadIdx.x; i < p.flux.n + 2; i += blockDim.x) sKn[i] = p.flux.kn[i];
     const int* gtab = static_cast<const int*>(p.flux.tab);
     for (int i = threadIdx.x; i < p.flux.ntab; i += blockDim.x) {
       const unsigned e = (unsigned)gtab[i];
@@ -276,7 +283,8 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
   __syncthreads();
   FluxView fx = p.flux;
   if (kSmemFlux) {
-    fx.kf = sKF;
+    fx.kn = sKn;
+    fx.seg = sSeg;
     fx.tab = sTab;
   }
   int* pre = sPre + 32 * warp;
@@ -598,25 +606,6 @@ __global__ void pixels_prepare_kernel(const double* __restrict__ dir, const doub
   }
 }
 
-// tab[c] = max{i : kappa_i <= kappa_0 + c * cell}: a start index for the flux search (M5)
-__global__ void flux_table_kernel(const double2* __restrict__ kf, int n, int* __restrict__ tab, int ntab,
-                                  double k0, double cell) {
-  for (int c = blockIdx.x * blockDim.x + threadIdx.x; c < ntab; c += gridDim.x * blockDim.x) {
-    const double x = k0 + (double)c * cell;
-    int lo = 0, hi = n - 1;
-    if (x >= kf[n - 1].x) {
-      tab[c] = n - 2;
-      continue;
-    }
-    while (hi - lo > 1) {
-      const int mid = (lo + hi) >> 1;
-      if (kf[mid].x <= x) lo = mid;
-      else hi = mid;
-    }
-    tab[c] = lo;
-  }
-}
-
 // ---------------------------------------------------------------- parity entry points
 struct RecordEmit {
   int64_t* bins;
@@ -697,12 +686,18 @@ int grid_for(int64_t work, int num_sms, int per_sm, int threads = kThreads) {
   return (int)std::max<int64_t>(blocks, 1);
 }
 
+// dynamic shared memory of the walk kernel (layout in mdnorm_walk_kernel)
+size_t walk_smem(const MdnParams& p, bool smem_flux, int threads) {
+  return (smem_flux ? sizeof(double4) * p.flux.n + sizeof(double) * ((p.flux.n + 3) & ~1) +
+                          sizeof(uint16_t) * ((p.flux.ntab + 1) & ~1)
+                    : 0) +
+         sizeof(int) * 32 * (threads / 32);
+}
+
 template <int kFlux, bool kStats, bool k3D>
 cudaError_t launch_walk(const MdnParams& p, int num_sms, cudaStream_t s) {
-  constexpr bool kSmemFlux = kFlux == 1;
   constexpr int threads = walk_threads(k3D);
-  const size_t smem = (kSmemFlux ? sizeof(double2) * (p.flux.n + 2) + sizeof(uint16_t) * ((p.flux.ntab + 1) & ~1) : 0) +
-                      sizeof(int) * 32 * (threads / 32);
+  const size_t smem = walk_smem(p, kFlux == 1, threads);
   auto k = mdnorm_walk_kernel<kFlux, kStats, k3D>;
   cudaError_t err = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (err != cudaSuccess) return err;
@@ -746,12 +741,6 @@ cudaError_t launch_pixels_prepare(const double* dir, const double* solid, double
   return cudaGetLastError();
 }
 
-cudaError_t launch_flux_table(const double2* kf, int n, int* tab, int ntab, double k0, double cell,
-                              cudaStream_t s) {
-  flux_table_kernel<<<grid_for(ntab, 148, 8), kThreads, 0, s>>>(kf, n, tab, ntab, k0, cell);
-  return cudaGetLastError();
-}
-
 cudaError_t launch_mdnorm(const MdnParams& p, const MatBlock& mb, int num_sms, cudaStream_t s) {
   if (p.plen == 0 || mb.nmat <= 0) return cudaSuccess;
   cudaError_t err = cudaMemsetAsync(p.ctr, 0, sizeof(DevCounters), s);
@@ -760,7 +749,13 @@ cudaError_t launch_mdnorm(const MdnParams& p, const MatBlock& mb, int num_sms, c
   if (err != cudaSuccess) return err;
   // 2-D slices (a single bin on the last axis, "lBins=1") merge two crossing streams
   const bool d3 = p.g.n[2] > 1;
-  const int mode = p.fviews ? 2 : (p.flux.n <= kFluxSmemMax ? 1 : 0);
+  // the flux table goes to shared memory when it fits one CTA (uint16 cell entries)
+  int dev = 0, smem_max = 0;
+  if ((err = cudaGetDevice(&dev)) != cudaSuccess) return err;
+  if ((err = cudaDeviceGetAttribute(&smem_max, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev)) != cudaSuccess)
+    return err;
+  const bool fits = p.flux.n <= kFluxSmemMax && walk_smem(p, true, walk_threads(d3)) <= (size_t)smem_max;
+  const int mode = p.fviews ? 2 : (fits ? 1 : 0);
 #define MDN_WALK_DISPATCH(F)                                                                    \
   if (d3) return p.stats ? launch_walk<F, true, true>(p, num_sms, s) : launch_walk<F, false, true>(p, num_sms, s); \
   return p.stats ? launch_walk<F, true, false>(p, num_sms, s) : launch_walk<F, false, false>(p, num_sms, s);

@@ -10,7 +10,7 @@ namespace mdn {
 constexpr int kMaxOps = 48;           // MDN_MAX_OPS
 constexpr int kMaxMats = 64;          // MDN_MAX_MATS
 constexpr int kRunsPerLaunch = 16;    // runs composed per MDNorm launch (batched API)
-constexpr int kFluxSmemMax = 4096;    // flux knots staged in shared memory (64 KB of double2)
+constexpr int kFluxSmemMax = 4096;    // flux knots staged in shared memory (44 B per knot: 180 KB)
 #ifndef MDN_PIECE_SEGS
 #define MDN_PIECE_SEGS 40  // measured: 40 > 24 > 16 (TOPAZ 200^3), ~flat on the CORELLI slab
 #endif
@@ -86,8 +86,6 @@ struct BinParams {
 // launchers (return the launch's cudaError_t)
 cudaError_t launch_pixels_prepare(const double* dir, const double* solid, double4* pix, int64_t npix,
                                   cudaStream_t s);
-cudaError_t launch_flux_table(const double2* kf, int n, int* tab, int ntab, double k0, double cell,
-                              cudaStream_t s);
 // MDNorm for shard pixels [p.p0, p.p0 + p.plen) x all matrices: cull (M1-M3) + piece walk (M3-M7).
 cudaError_t launch_mdnorm(const MdnParams& p, const MatBlock& mb, int num_sms, cudaStream_t s);
 cudaError_t launch_binmd(const BinParams& p, const MatBlock& mb, int num_sms, cudaStream_t s);
