@@ -273,127 +273,6 @@ __device__ __forceinline__ void cursor_init(AxisCursor& c, const GridC& g, int a
   c.nk = s.cnt > 0 ? dmul(dadd(g.lo[a], dmul(c.jd, g.w[a])), c.r) : CUDART_INF;
 }
 
-// ------------------------------------------------------------------------------ M4-M7
-// Walk the part [lo_k, hi_k] of a clipped trajectory, where lo_k and hi_k are members of the
-// trajectory's list L (its clip endpoints or plane crossings): a 3-way streaming merge of the
-// per-axis monotone crossing sequences strictly inside (lo_k, hi_k) (replaces the paper's sort,
-// P:115, and the GPU comb sort, with no buffer), flux at each list entry (M5), midpoint
-// bin of every positive-length segment (M6) and emit(b, (F(k2) - F(k1)) * omega_c) (M7).
-// Splitting L at any of its members leaves the set of segments unchanged, which is what lets
-// the production kernel cut long trajectories into balanced pieces.  The merge step is written
-// with selects only (no per-axis branches) so that the lanes of a warp stay converged.
-// Returns n_seg; *ncross receives the number of crossings strictly inside (lo_k, hi_k).
-template <bool k3D, typename TabT = int, class Emit>
-__device__ __forceinline__ int traj_walk(const GridC& g, const FluxView& fx, double v0, double v1,
-                                         double v2, double lo_k, double hi_k, double omega_c,
-                                         Emit& emit, int* ncross) {
-  // k3D = false: the last axis has a single bin (2-D slice), so it never has a crossing
-  AxisCursor c0, c1, c2;
-  cursor_init(c0, g, 0, v0, lo_k, hi_k);
-  cursor_init(c1, g, 1, v1, lo_k, hi_k);
-  if (k3D) {
-    cursor_init(c2, g, 2, v2, lo_k, hi_k);
-  } else {
-    c2.cnt = 0;
-    c2.nk = CUDART_INF;
-    c2.jd = c2.stepd = c2.r = 0.0;
-  }
-  const int total = c0.cnt + c1.cnt + c2.cnt;
-  *ncross = total;
-  double k1 = lo_k, F1 = flux_at<TabT>(fx, lo_k);
-  int nseg = 0;
-  int left = total;
-  // next entry of L: the smallest pending crossing (ties: lowest axis first; equal values give
-  // a skipped zero-length segment, so the order among ties never matters), then hi_k
-  auto next = [&]() -> double {
-    if (left == 0) return hi_k;
-    --left;
-    if (!k3D) {  // 2-D slice: two streams
-#if MDN_MERGE2D_SELECT
-      const bool p0 = c0.nk <= c1.nk;
-      const double k = p0 ? c0.nk : c1.nk;
-      const double jd = p0 ? c0.jd + c0.stepd : c1.jd + c1.stepd;
-      const int cnt = (p0 ? c0.cnt : c1.cnt) - 1;
-      const double nk = cnt > 0 ? dmul(dadd(p0 ? g.lo[0] : g.lo[1], dmul(jd, p0 ? g.w[0] : g.w[1])), p0 ? c0.r : c1.r)
-                                : CUDART_INF;
-      c0.jd = p0 ? jd : c0.jd;
-      c0.cnt = p0 ? cnt : c0.cnt;
-      c0.nk = p0 ? nk : c0.nk;
-      c1.jd = p0 ? c1.jd : jd;
-      c1.cnt = p0 ? c1.cnt : cnt;
-      c1.nk = p0 ? c1.nk : nk;
-      return k;
-#else
-      if (c0.nk <= c1.nk) {
-        const double k = c0.nk;
-        c0.jd += c0.stepd;
-        --c0.cnt;
-        c0.nk = c0.cnt > 0 ? dmul(dadd(g.lo[0], dmul(c0.jd, g.w[0])), c0.r) : CUDART_INF;
-        return k;
-      }
-      const double k = c1.nk;
-      c1.jd += c1.stepd;
-      --c1.cnt;
-      c1.nk = c1.cnt > 0 ? dmul(dadd(g.lo[1], dmul(c1.jd, g.w[1])), c1.r) : CUDART_INF;
-      return k;
-#endif
-    }
-    // three streams, selects only: advance the chosen axis with one plane evaluation
-    const bool s01 = c1.nk < c0.nk;
-    const double m01 = s01 ? c1.nk : c0.nk;
-    const bool s2 = c2.nk < m01;
-    const bool p0 = !s2 && !s01, p1 = !s2 && s01;
-    const double k = s2 ? c2.nk : m01;
-    const double jd = (p0 ? c0.jd + c0.stepd : (p1 ? c1.jd + c1.stepd : c2.jd + c2.stepd));
-    const int cnt = (p0 ? c0.cnt : (p1 ? c1.cnt : c2.cnt)) - 1;
-    const double lo = p0 ? g.lo[0] : (p1 ? g.lo[1] : g.lo[2]);
-    const double w = p0 ? g.w[0] : (p1 ? g.w[1] : g.w[2]);
-    const double r = p0 ? c0.r : (p1 ? c1.r : c2.r);
-    const double nk = cnt > 0 ? dmul(dadd(lo, dmul(jd, w)), r) : CUDART_INF;
-    if (p0) { c0.jd = jd; c0.cnt = cnt; c0.nk = nk; }
-    if (p1) { c1.jd = jd; c1.cnt = cnt; c1.nk = nk; }
-    if (s2) { c2.jd = jd; c2.cnt = cnt; c2.nk = nk; }
-    return k;
-  };
-  // segment (k1, k2) if it has positive length: midpoint bin (M6) and value (M7)
-  auto segment = [&](double k2, double F2) {
-    if (k2 > k1) {
-      const double km = dmul(0.5, dadd(k1, k2));
-      const double t0 = dmul(dsub(dmul(km, v0), g.lo[0]), g.s[0]);
-      const double t1 = dmul(dsub(dmul(km, v1), g.lo[1]), g.s[1]);
-      const double t2 = dmul(dsub(dmul(km, v2), g.lo[2]), g.s[2]);
-      // for finite t, (0 <= t < n) <=> (unsigned)floor(t) < n (floor saturates, -0 -> 0); the
-      // walk only sees finite v (the cull drops non-finite directions)
-      const int i0 = __double2int_rd(t0), i1 = __double2int_rd(t1), i2 = __double2int_rd(t2);
-      if ((unsigned)i0 < (unsigned)g.n[0] && (unsigned)i1 < (unsigned)g.n[1] && (unsigned)i2 < (unsigned)g.n[2]) {
-        emit(i0 + g.n[0] * (i1 + g.n[1] * i2), dmul(dsub(F2, F1), omega_c));
-        ++nseg;
-      }
-      k1 = k2;
-      F1 = F2;
-    }
-  };
-  // L has total + 1 entries after lo_k.  3-D: two at a time, so that their flux look-ups (the
-  // longest dependency chain) are independent and overlap; 2-D slices (two streams, fewer live
-  // registers) measured faster one at a time.
-  int rem = total + 1;
-  if (k3D) {
-    for (; rem >= 2; rem -= 2) {
-      const double ka = next();
-      const double kb = next();
-      const double Fa = flux_at<TabT>(fx, ka);
-      const double Fb = flux_at<TabT>(fx, kb);
-      segment(ka, Fa);
-      segment(kb, Fb);
-    }
-  }
-  for (; rem >= 1; --rem) {
-    const double ka = next();
-    segment(ka, flux_at<TabT>(fx, ka));
-  }
-  return nseg;
-}
-
 // ------------------------------------------------------------------------------ B2-B3
 // Bin of event Q (fp32 input widened to fp64) under N: x_a = ((N_a0 q0 + N_a1 q1) + N_a2 q2),
 // t_a = (x_a - lo_a) s_a, inside iff 0 <= t_a < n_a for every a.  -1 = outside.

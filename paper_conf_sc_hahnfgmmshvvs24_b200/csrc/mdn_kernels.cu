@@ -15,6 +15,7 @@
 #include <algorithm>
 
 #include "mdn_kernels.cuh"
+#include "mdn_walk.cuh"
 
 namespace mdn {
 
@@ -32,6 +33,13 @@ namespace {
 #ifndef MDN_WALK_MINB
 #define MDN_WALK_MINB 1
 #endif
+// walk warps claim hitters kWalkChunk at a time into a per-warp ring of kWalkRing entries
+#ifndef MDN_WALK_CHUNK
+#define MDN_WALK_CHUNK 8
+#endif
+constexpr int kWalkChunk = MDN_WALK_CHUNK;
+constexpr int kWalkRing = 64;  // >= 31 + the largest claim (32), a power of two
+static_assert(kWalkChunk >= 1 && kWalkChunk <= 32, "walk claim size");
 constexpr int kThreads = 256;
 constexpr int walk_threads(bool k3D) { return k3D ? MDN_WALK_THREADS_3D : MDN_WALK_THREADS; }
 constexpr unsigned kFull = 0xffffffffu;
@@ -265,12 +273,13 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int nwarps = blockDim.x >> 5;
   // shared layout: interval records (n double4) | knots (n + 2, even) | cell table (uint16, even)
-  // | per-warp prefix sums
+  // | per-warp prefix sums (32 int) | per-warp hitter rings (kWalkRing unsigned)
   const int n_kn = kSmemFlux ? (p.flux.n + 3) & ~1 : 0;
   double4* sSeg = wsm;
   double* sKn = reinterpret_cast<double*>(sSeg + (kSmemFlux ? p.flux.n : 0));
   uint16_t* sTab = reinterpret_cast<uint16_t*>(sKn + n_kn);
   int* sPre = reinterpret_cast<int*>(sTab + (kSmemFlux ? (p.flux.ntab + 1) & ~1 : 0));
+  unsigned* sRing = reinterpret_cast<unsigned*>(sPre + 32 * nwarps);
   if (kSmemFlux) {
     for (int i = threadIdx.x; i < p.flux.n; i += blockDim.x) sSeg[i] = p.flux.seg[i];
     for (int i = threadIdx.x; i < p.flux.n + 2; i += blockDim.x) sKn[i] = p.flux.kn[i];
@@ -288,63 +297,99 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
     fx.tab = sTab;
   }
   int* pre = sPre + 32 * warp;
-  (void)nwarps;
   AtomicEmit emit{p.norm};
   const unsigned nhit = *(volatile unsigned*)&p.ctr->nhit;
   unsigned long long c_seg = 0;
+  // Per-warp queue of hitters (ring of kWalkRing indices; the head hitter may be partly
+  // consumed: `skip` of its pieces are done) holding `qpieces` pieces.  Each round hands the next
+  // 32 pieces of the queue to the 32 lanes, which walk them to completion together (so the piece
+  // set-up -- divisions, per-axis ranges, first flux look-up -- runs converged).  The queue is
+  // topped up by claiming kWalkChunk hitters at a time from the global cursor, so rounds are full
+  // across hitter boundaries and the end-of-kernel imbalance is one small chunk.
+  unsigned* ring = sRing + 2 * kWalkRing * warp;  // hitter indices
+  int* ringP = reinterpret_cast<int*>(ring + kWalkRing);  // their piece counts
+  unsigned head = 0, nq = 0;
+  int skip = 0, qpieces = 0;
+  bool more = true;
+  const unsigned tail = 4u * 32u * gridDim.x * (unsigned)nwarps;
+  unsigned chunk = nhit > tail ? 32u : (unsigned)kWalkChunk;
   for (;;) {
-    unsigned b = 0;
-    if (lane == 0) b = atomicAdd(&p.ctr->batch, 1u);
-    b = __shfl_sync(kFull, b, 0);
-    const unsigned h0 = b * 32u;
-    if (h0 >= nhit) break;
-    const unsigned hl = h0 + lane;
-    int P = hl < nhit ? p.hit[hl].P : 0;
-    // inclusive warp scan of piece counts
-    int incl = P;
+    while (qpieces < 32 && more) {
+      unsigned b = 0;
+      if (lane == 0) b = atomicAdd(&p.ctr->claimed, chunk);
+      b = __shfl_sync(kFull, b, 0);
+      if (b >= nhit) {
+        more = false;
+        break;
+      }
+      const unsigned nnew = min(chunk, nhit - b);
+      // large claims (hitter locality, fewer atomics) until the last few claims per warp, then
+      // small ones so that the warps finish together
+      chunk = nhit - b > tail ? 32u : (unsigned)kWalkChunk;
+      int P = 0;
+      if ((unsigned)lane < nnew) {
+        P = p.hit[b + lane].P;
+        ring[(head + nq + lane) & (kWalkRing - 1)] = b + lane;
+        ringP[(head + nq + lane) & (kWalkRing - 1)] = P;
+      }
+      nq += nnew;
+      qpieces += __reduce_add_sync(kFull, P);
+      __syncwarp();
+    }
+    if (qpieces == 0) break;
+    // pieces of the first (up to) 32 queued hitters: inclusive scan of their remaining counts
+    const bool inq = (unsigned)lane < nq;
+    int incl = inq ? ringP[(head + lane) & (kWalkRing - 1)] - (lane == 0 ? skip : 0) : 0;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
       const int y = __shfl_up_sync(kFull, incl, o);
       if (lane >= o) incl += y;
     }
     pre[lane] = incl;
-    const int total = __shfl_sync(kFull, incl, 31);
     __syncwarp();
-    // round-synchronous: the lanes start their pieces together, so the piece set-up (divisions,
-    // per-axis ranges, first flux lookup) runs converged
-    for (int q0 = 0; q0 < total; q0 += 32) {
-      const int q = q0 + lane;
-      if (q < total) {
-        // owner hitter: first l with pre[l] > q
-        int l = 0;
+    const int nr = min(qpieces, 32);
+    unsigned myh = 0;
+    int mypi = 0;
+    if (lane < nr) {
+      int l = 0;  // owner: first queued hitter l with pre[l] > lane
 #pragma unroll
-        for (int s = 16; s > 0; s >>= 1)
-          if (pre[l + s - 1] <= q) l += s;
-        const int pi = q - (l ? pre[l - 1] : 0);
-        const Hitter& h = p.hit[h0 + l];
-        const double v0 = h.v0, v1 = h.v1, v2 = h.v2;
-        const int A = h.A & 3;
-        double lo_k = h.kin, hi_k = h.kout;
-        if (h.P > 1) {
-          const double vA = A == 0 ? v0 : (A == 1 ? v1 : v2);
-          const double rA = ddiv(1.0, vA);
-          if (pi > 0) lo_k = plane_k(p.g, A, h.jA + pi * h.stepG, rA);
-          if (pi < h.P - 1) hi_k = plane_k(p.g, A, h.jA + (pi + 1) * h.stepG, rA);
-        }
-        int nc;
-        int ns;
-        if (kFlux == 1) {
-          ns = traj_walk<k3D, uint16_t>(p.g, fx, v0, v1, v2, lo_k, hi_k, h.oc, emit, &nc);
-        } else if (kFlux == 2) {
-          const FluxView fv = p.fviews[h.A >> 2];
-          ns = traj_walk<k3D, int>(p.g, fv, v0, v1, v2, lo_k, hi_k, h.oc, emit, &nc);
-        } else {
-          ns = traj_walk<k3D, int>(p.g, fx, v0, v1, v2, lo_k, hi_k, h.oc, emit, &nc);
-        }
-        if (kStats) c_seg += ns;
-      }
-      __syncwarp();
+      for (int s = 16; s > 0; s >>= 1)
+        if (pre[l + s - 1] <= lane) l += s;
+      myh = ring[(head + l) & (kWalkRing - 1)];
+      mypi = lane - (l ? pre[l - 1] : 0) + (l == 0 ? skip : 0);
     }
+    // advance the queue past the nr pieces handed out
+    const int k = __popc(__ballot_sync(kFull, inq && incl <= nr));  // hitters fully consumed
+    const int kpre = k ? __shfl_sync(kFull, incl, (k - 1) & 31) : 0;
+    skip = k ? nr - kpre : skip + nr;
+    head += k;
+    nq -= k;
+    qpieces -= nr;
+    __syncwarp();
+    if (lane < nr) {
+      const Hitter& h = p.hit[myh];
+      const double v0 = h.v0, v1 = h.v1, v2 = h.v2;
+      const int A = h.A & 3;
+      double lo_k = h.kin, hi_k = h.kout;
+      if (h.P > 1) {
+        const double vA = A == 0 ? v0 : (A == 1 ? v1 : v2);
+        const double rA = ddiv(1.0, vA);
+        if (mypi > 0) lo_k = plane_k(p.g, A, h.jA + mypi * h.stepG, rA);
+        if (mypi < h.P - 1) hi_k = plane_k(p.g, A, h.jA + (mypi + 1) * h.stepG, rA);
+      }
+      int nc;
+      int ns;
+      if (kFlux == 1) {
+        ns = traj_walk<k3D, uint16_t>(p.g, fx, v0, v1, v2, lo_k, hi_k, h.oc, emit, &nc);
+      } else if (kFlux == 2) {
+        const FluxView fv = p.fviews[h.A >> 2];
+        ns = traj_walk<k3D, int>(p.g, fv, v0, v1, v2, lo_k, hi_k, h.oc, emit, &nc);
+      } else {
+        ns = traj_walk<k3D, int>(p.g, fx, v0, v1, v2, lo_k, hi_k, h.oc, emit, &nc);
+      }
+      if (kStats) c_seg += ns;
+    }
+    __syncwarp();
   }
   if (kStats) flush_counter(p.stats + 3, c_seg);
 }
@@ -691,7 +736,7 @@ size_t walk_smem(const MdnParams& p, bool smem_flux, int threads) {
   return (smem_flux ? sizeof(double4) * p.flux.n + sizeof(double) * ((p.flux.n + 3) & ~1) +
                           sizeof(uint16_t) * ((p.flux.ntab + 1) & ~1)
                     : 0) +
-         sizeof(int) * 32 * (threads / 32);
+         (sizeof(int) * 32 + 2 * sizeof(unsigned) * kWalkRing) * (threads / 32);
 }
 
 template <int kFlux, bool kStats, bool k3D>

@@ -48,7 +48,7 @@ struct alignas(16) Hitter {
 
 struct DevCounters {
   unsigned int nhit;     // hitters written by the cull kernel
-  unsigned int batch;    // warp batches claimed by the walk kernel
+  unsigned int claimed;  // hitters claimed by the walk kernel's warps
   unsigned int pad[2];
 };
 
