@@ -440,15 +440,15 @@ mdn_status mdnorm_set_instrument(mdn_grid* g, int64_t npix, const double* dir, c
 namespace {
 
 // Host image of one flux table (M5, see flux_at in mdn_device.cuh): knots kappa_i + two +inf
-// pads; per interval (Phi_i, dPhi_i, y_i, dk_i) with dPhi_i = Phi_{i+1} - Phi_i, dk_i =
-// kappa_{i+1} - kappa_i, y_i = 1 / dk_i (IEEE double, the same roundings as the device); and the
-// cell table over U(x) = (x - kappa_0) * inv_cell: entry c = s_c = max{i : U_i < c}, flagged
-// when cell c holds more than three knots, when s_c does not exist (c = 0) or when c + 1 > U_{n-1}.
-// max(2n, range / (2.9 min spacing)) cells, at most 2^22.  This file is compiled with -ffp-contract=off, so U_i is exactly the
-// device's dmul(dsub(x, kappa_0), inv_cell).
+// pads; per interval ka_i = (kappa_i, Phi_i), kb_i = (dPhi_i, y_i) with dPhi_i = Phi_{i+1} -
+// Phi_i, y_i = 1 / (kappa_{i+1} - kappa_i) (IEEE double, the same roundings as the device); and
+// the cell table over U(x) = (x - kappa_0) * inv_cell: entry c = s_c = max{i : U_i < c}, flagged
+// when cell c holds more than three knots, when s_c does not exist (c = 0) or when c + 1 >
+// U_{n-1}.  max(4n, range / (2.9 min spacing)) cells, at most 2^22.  This file is compiled with
+// -ffp-contract=off, so U_i is exactly the device's dmul(dsub(x, kappa_0), inv_cell).
 struct HostFluxTable {
   std::vector<double> kn;
-  std::vector<double4> seg;
+  std::vector<double2> ka, kb;
   std::vector<int> tab;
   double k_first, F_first, k_last, F_last, inv_cell;
   int n, ntab;
@@ -464,19 +464,22 @@ mdn_status build_flux_table(const double* hk, const double* hF, int64_t n, HostF
   t.kn.assign(hk, hk + n);
   t.kn.push_back(HUGE_VAL);
   t.kn.push_back(HUGE_VAL);
-  t.seg.assign((size_t)n, make_double4(0.0, 0.0, 0.0, 0.0));
+  t.ka.assign((size_t)n, make_double2(0.0, 0.0));
+  t.kb.assign((size_t)n, make_double2(0.0, 0.0));
   for (int64_t i = 0; i + 1 < n; ++i) {
     const double dk = hk[i + 1] - hk[i];
     const double dF = hF[i + 1] - hF[i];
     if (!std::isfinite(dk) || !std::isfinite(dF) || !std::isfinite(1.0 / dk))
       return fail(MDN_EINVAL, "flux table interval %lld overflows", (long long)i);
-    t.seg[i] = make_double4(hF[i], dF, 1.0 / dk, dk);
+    t.ka[i] = make_double2(hk[i], hF[i]);
+    t.kb[i] = make_double2(dF, 1.0 / dk);
   }
-  // cells narrower than 3 x the smallest knot spacing hold at most 3 knots (all fast)
+  // cells narrower than 3 x the smallest knot spacing hold at most 3 knots (all fast); four cells
+  // per knot make a knot at or below x in x's own cell rare (the one-probe look-up)
   double hmin = HUGE_VAL;
   for (int64_t i = 0; i + 1 < n; ++i) hmin = std::min(hmin, hk[i + 1] - hk[i]);
   const double want = std::ceil((hk[n - 1] - hk[0]) / (2.9 * hmin));
-  const int ntab = (int)std::min<double>(std::max<double>(2.0 * (double)n, want), (double)(1 << 22));
+  const int ntab = (int)std::min<double>(std::max<double>(4.0 * (double)n, want), (double)(1 << 22));
   t.inv_cell = (double)ntab / (hk[n - 1] - hk[0]);
   if (!std::isfinite(t.inv_cell)) return fail(MDN_EINVAL, "flux table k range too small");
   std::vector<double> U((size_t)n);
@@ -530,27 +533,30 @@ mdn_status mdnorm_set_flux_tables(mdn_grid* g, int32_t ntables, const int64_t* o
                                tabs[t])) != MDN_OK)
       return st;
   // concatenate into one allocation: every table's knots (padded to an even count, so the
-  // interval records stay 16-byte aligned), then every table's interval records; the cell
-  // tables in a second allocation; one FluxView per table
-  size_t nkn = 0, nseg = 0, ntb = 0;
+  // interval records stay 16-byte aligned), then every table's ka records, then every table's kb
+  // records; the cell tables in a second allocation; one FluxView per table
+  size_t nkn = 0, nrec = 0, ntb = 0;
   for (auto& t : tabs) {
     nkn += (t.kn.size() + 1) & ~size_t(1);
-    nseg += t.seg.size();
+    nrec += t.ka.size();
     ntb += t.tab.size();
   }
-  std::vector<double> all(nkn + 4 * nseg, 0.0);
+  std::vector<double> all(nkn + 4 * nrec, 0.0);
   std::vector<int> all_tab;
   all_tab.reserve(ntb);
-  std::vector<size_t> kn_off, seg_off, tb_off;
-  size_t o = 0, so = nkn;
+  std::vector<size_t> kn_off, ka_off, kb_off, tb_off;
+  size_t o = 0, ao = nkn, bo = nkn + 2 * nrec;
   for (auto& t : tabs) {
     kn_off.push_back(o);
-    seg_off.push_back(so);
+    ka_off.push_back(ao);
+    kb_off.push_back(bo);
     tb_off.push_back(all_tab.size());
     std::copy(t.kn.begin(), t.kn.end(), all.begin() + o);
-    std::memcpy(all.data() + so, t.seg.data(), sizeof(double4) * t.seg.size());
+    std::memcpy(all.data() + ao, t.ka.data(), sizeof(double2) * t.ka.size());
+    std::memcpy(all.data() + bo, t.kb.data(), sizeof(double2) * t.kb.size());
     o += (t.kn.size() + 1) & ~size_t(1);
-    so += 4 * t.seg.size();
+    ao += 2 * t.ka.size();
+    bo += 2 * t.kb.size();
     all_tab.insert(all_tab.end(), t.tab.begin(), t.tab.end());
   }
   double* d = nullptr;
@@ -566,7 +572,8 @@ mdn_status mdnorm_set_flux_tables(mdn_grid* g, int32_t ntables, const int64_t* o
     mdn::FluxView& v = hv[t];
     v = mdn::FluxView{};
     v.kn = d + kn_off[t];
-    v.seg = reinterpret_cast<const double4*>(d + seg_off[t]);
+    v.ka = reinterpret_cast<const double2*>(d + ka_off[t]);
+    v.kb = reinterpret_cast<const double2*>(d + kb_off[t]);
     v.tab = tab + tb_off[t];
     v.k_first = tabs[t].k_first;
     v.F_first = tabs[t].F_first;

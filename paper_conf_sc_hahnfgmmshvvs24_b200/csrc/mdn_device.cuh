@@ -100,9 +100,10 @@ __device__ __forceinline__ bool compose_binmd(const double* UB, const double* S,
 // F(x): clamp outside, else i = max{i : kappa_i <= x} and
 //   Phi_i + (Phi_{i+1} - Phi_i) * ((x - kappa_i) / (kappa_{i+1} - kappa_i)).
 //
-// Per interval the table stores (Phi_i, dPhi_i, y_i, dk_i) with dPhi_i = RN(Phi_{i+1} - Phi_i),
-// dk_i = RN(kappa_{i+1} - kappa_i) (the same roundings as the formula) and y_i = RN(1 / dk_i).
-// The correctly rounded quotient a / dk_i (a = RN(x - kappa_i)) is then
+// Per interval the table stores ka_i = (kappa_i, Phi_i) and kb_i = (dPhi_i, y_i) with dPhi_i =
+// RN(Phi_{i+1} - Phi_i) and y_i = RN(1 / dk_i), dk_i = RN(kappa_{i+1} - kappa_i) (the same
+// roundings as the formula; dk_i is recomputed from the knots).  The correctly rounded quotient
+// a / dk_i (a = RN(x - kappa_i)) is then
 //   q = RN(a y_i);  r = a - q dk_i (exact, one FMA);  q' = RN(q + r y_i)   (one FMA)
 // -- Markstein's theorem: y within half an ulp of 1/b and q within one ulp of a/b make r exact
 // and q' = RN(a/b) (no overflow / underflow here: 0 <= a < dk, both normal or zero).  Three
@@ -112,16 +113,25 @@ __device__ __forceinline__ bool compose_binmd(const double* UB, const double* S,
 // Search: U(x) = RN(RN(x - kappa_0) * inv_cell) is monotone non-decreasing in x, and the host
 // evaluates the same expression U_i = U(kappa_i).  For x with floor(U(x)) = c:
 //   every knot with U_i < c is < x, and every knot with U_i >= c + 1 is > x,
-// so i = s_c + #{probes kappa_{s_c+1..s_c+3} <= x} with s_c = max{i : U_i < c}, provided cell
-// c holds at most three knots (#{i : floor(U_i) = c} <= 3) and c + 1 <= U_{n-1} (then x <
-// kappa_{n-1}, no clamp).  Cells failing that (and c = 0, x outside the table) are flagged and
-// take the general path: clamps and a bisection.  Two (+inf) pad knots keep the probes in bounds.
+// so with s_c = max{i : U_i < c}, i is s_c plus the number of knots of cell c that are <= x:
+// probe kappa_{s_c+1}, kappa_{s_c+2}, ... until the first knot > x (which is kappa_{i+1}, the
+// knot dk_i needs).  The common case -- no knot of cell c at or below x -- needs one probe, and
+// the interval records are loaded alongside it; cells are four per knot (or narrower), so a
+// probe finds a knot <= x for ~1/8 of the look-ups.  Cells with more than three knots (and c =
+// 0, x outside the table, or c + 1 > U_{n-1}) are flagged and take the general path: clamps and
+// a bisection.  Two (+inf) pad knots keep the probes in bounds.
+//
+// Shared-memory layout (bank conflicts of random look-ups, measured: profiles/): knots as a
+// dense double array (8-byte probes over 16 bank pairs) and the two records as separate
+// 16-byte-strided double2 arrays (all 8 sixteen-byte bank groups), instead of one 32-byte record
+// per interval (which uses only 4 of the 8 groups).
 constexpr unsigned kFluxDense32 = 1u << 30;  // flag bit in an int32 table entry
 constexpr unsigned kFluxDense16 = 1u << 15;  // flag bit in a uint16 (shared-memory) entry
 
 struct FluxView {
   const double* kn;    // kappa_i: n knots + 2 (+inf) pads
-  const double4* seg;  // per interval i < n - 1: (Phi_i, dPhi_i, y_i, dk_i); n entries
+  const double2* ka;   // per interval i < n - 1: (kappa_i, Phi_i); n entries
+  const double2* kb;   // per interval i < n - 1: (dPhi_i, y_i); n entries
   const void* tab;     // ntab cell entries: int32 (global) or uint16 (shared-memory copy)
   double k_first, F_first, k_last, F_last, inv_cell;
   int n, ntab;
@@ -132,14 +142,14 @@ __device__ __forceinline__ unsigned tab_entry(const FluxView& f, int c) {
   return (unsigned)static_cast<const TabT*>(f.tab)[c];
 }
 
-// Phi_i + dPhi_i * RN((x - kappa_i) / dk_i) for kappa_i <= x < kappa_{i+1}
-__device__ __forceinline__ double flux_interp(const FluxView& f, int i, double x) {
-  const double4 s = f.seg[i];
-  const double a = dsub(x, f.kn[i]);
-  const double q = dmul(a, s.z);
-  const double r = __fma_rn(-q, s.w, a);
-  const double t = __fma_rn(r, s.z, q);
-  return dadd(s.x, dmul(s.y, t));
+// Phi_i + dPhi_i * RN((x - kappa_i) / dk_i) for kappa_i <= x < kappa_{i+1} = kn1
+__device__ __forceinline__ double flux_interp(double x, double2 a, double2 b, double kn1) {
+  const double d = dsub(x, a.x);
+  const double dk = dsub(kn1, a.x);
+  const double q = dmul(d, b.y);
+  const double r = __fma_rn(-q, dk, d);
+  const double t = __fma_rn(r, b.y, q);
+  return dadd(a.y, dmul(b.x, t));
 }
 
 __device__ __forceinline__ double flux_general(const FluxView& f, double x) {
@@ -152,7 +162,7 @@ __device__ __forceinline__ double flux_general(const FluxView& f, double x) {
     if (f.kn[lo + half] <= x) lo += half;
     len -= half;
   }
-  return flux_interp(f, lo, x);
+  return flux_interp(x, f.ka[lo], f.kb[lo], f.kn[lo + 1]);
 }
 
 template <typename TabT = int>
@@ -164,8 +174,18 @@ __device__ __forceinline__ double flux_at(const FluxView& f, double x) {
   const int c = __double2int_rd(dmul(dsub(x, f.k_first), f.inv_cell));
   const unsigned e = (unsigned)c < (unsigned)f.ntab ? tab_entry<TabT>(f, c) : flag;
   if (e & flag) return flux_general(f, x);
-  const int i = (int)e + (f.kn[e + 1] <= x ? 1 : 0) + (f.kn[e + 2] <= x ? 1 : 0) + (f.kn[e + 3] <= x ? 1 : 0);
-  return flux_interp(f, i, x);
+  int i = (int)e;
+  double kn1 = f.kn[i + 1];
+  double2 a = f.ka[i], b = f.kb[i];
+  if (kn1 <= x) {  // a knot of cell c lies at or below x (at most three)
+    do {
+      ++i;
+      kn1 = f.kn[i + 1];
+    } while (kn1 <= x);
+    a = f.ka[i];
+    b = f.kb[i];
+  }
+  return flux_interp(x, a, b, kn1);
 }
 
 // ------------------------------------------------------------------------------ M1-M2

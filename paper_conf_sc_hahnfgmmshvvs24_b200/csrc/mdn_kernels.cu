@@ -272,16 +272,21 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
   extern __shared__ double4 wsm[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int nwarps = blockDim.x >> 5;
-  // shared layout: interval records (n double4) | knots (n + 2, even) | cell table (uint16, even)
-  // | per-warp prefix sums (32 int) | per-warp hitter rings (kWalkRing unsigned)
+  // shared layout: interval records ka, kb (n double2 each) | knots (n + 2, even) | cell table
+  // (uint16, even) | per-warp prefix sums (32 int) | per-warp hitter rings (kWalkRing unsigned)
+  const int n_rec = kSmemFlux ? p.flux.n : 0;
   const int n_kn = kSmemFlux ? (p.flux.n + 3) & ~1 : 0;
-  double4* sSeg = wsm;
-  double* sKn = reinterpret_cast<double*>(sSeg + (kSmemFlux ? p.flux.n : 0));
+  double2* sKa = reinterpret_cast<double2*>(wsm);
+  double2* sKb = sKa + n_rec;
+  double* sKn = reinterpret_cast<double*>(sKb + n_rec);
   uint16_t* sTab = reinterpret_cast<uint16_t*>(sKn + n_kn);
   int* sPre = reinterpret_cast<int*>(sTab + (kSmemFlux ? (p.flux.ntab + 1) & ~1 : 0));
   unsigned* sRing = reinterpret_cast<unsigned*>(sPre + 32 * nwarps);
   if (kSmemFlux) {
-    for (int i = threadIdx.x; i < p.flux.n; i += blockDim.x) sSeg[i] = p.flux.seg[i];
+    for (int i = threadIdx.x; i < p.flux.n; i += blockDim.x) {
+      sKa[i] = p.flux.ka[i];
+      sKb[i] = p.flux.kb[i];
+    }
     for (int i = threadIdx.x; i < p.flux.n + 2; i += blockDim.x) sKn[i] = p.flux.kn[i];
     const int* gtab = static_cast<const int*>(p.flux.tab);
     for (int i = threadIdx.x; i < p.flux.ntab; i += blockDim.x) {
@@ -293,7 +298,8 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
   FluxView fx = p.flux;
   if (kSmemFlux) {
     fx.kn = sKn;
-    fx.seg = sSeg;
+    fx.ka = sKa;
+    fx.kb = sKb;
     fx.tab = sTab;
   }
   int* pre = sPre + 32 * warp;
@@ -733,7 +739,7 @@ int grid_for(int64_t work, int num_sms, int per_sm, int threads = kThreads) {
 
 // dynamic shared memory of the walk kernel (layout in mdnorm_walk_kernel)
 size_t walk_smem(const MdnParams& p, bool smem_flux, int threads) {
-  return (smem_flux ? sizeof(double4) * p.flux.n + sizeof(double) * ((p.flux.n + 3) & ~1) +
+  return (smem_flux ? 2 * sizeof(double2) * p.flux.n + sizeof(double) * ((p.flux.n + 3) & ~1) +
                           sizeof(uint16_t) * ((p.flux.ntab + 1) & ~1)
                     : 0) +
          (sizeof(int) * 32 + 2 * sizeof(unsigned) * kWalkRing) * (threads / 32);

@@ -10,7 +10,7 @@ namespace mdn {
 constexpr int kMaxOps = 48;           // MDN_MAX_OPS
 constexpr int kMaxMats = 64;          // MDN_MAX_MATS
 constexpr int kRunsPerLaunch = 16;    // runs composed per MDNorm launch (batched API)
-constexpr int kFluxSmemMax = 4096;    // flux knots staged in shared memory (44 B per knot: 180 KB)
+constexpr int kFluxSmemMax = 4096;    // flux knots staged in shared memory (48 B per knot: 196 KB)
 #ifndef MDN_PIECE_SEGS
 #define MDN_PIECE_SEGS 40  // measured: 40 > 24 > 16 (TOPAZ 200^3), ~flat on the CORELLI slab
 #endif
