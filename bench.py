@@ -64,6 +64,18 @@ def ncu_traffic():
     return {}
 
 
+def atomic_roof():
+    """Measured fp64 red.global.add rate into an L2-resident histogram (tools/roofs.cu on a B200
+    of this pool, committed as profiles/rNN_roofs.json; the newest file wins)."""
+    import glob
+    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "r*_roofs.json")))
+    if not files:
+        return None, None
+    with open(files[-1]) as f:
+        r = json.load(f)
+    return float(r["atomics_per_s"]["corelli_600x600"]["red_f64_random"]), os.path.relpath(files[-1], ROOT)
+
+
 # ----------------------------------------------------------------------------- clocks
 
 
@@ -325,12 +337,21 @@ def run_ours(args, rank, world, local_rank):
     md_traffic = None
     if "mdnorm_cull_kernel" in traffic and "mdnorm_walk_kernel" in traffic:
         md_traffic = traffic["mdnorm_cull_kernel"] + traffic["mdnorm_walk_kernel"]
-    kernels["mdnorm"] = {"kernels": "mdnorm_cull_kernel + mdnorm_walk_kernel",
-                         "bound": "alu", "achieved": md_ops / t / 1e12, "peak": fp64_peak,
-                         "unit": "TFLOP/s", "frac": md_ops / t / 1e12 / fp64_peak,
-                         "traffic": md_traffic, "ms": ph_ms["mdnorm"], "ops_per_launch": md_ops,
-                         "peak_note": f"fp64 non-fused ops at {sm_max:.0f} MHz (148 SM x 64 lanes), "
-                                      "DESIGN.md §4"}
+    alu = {"bound": "alu", "achieved": md_ops / t / 1e12, "peak": fp64_peak, "unit": "TFLOP/s",
+           "frac": md_ops / t / 1e12 / fp64_peak,
+           "peak_note": f"fp64 non-fused ops at {sm_max:.0f} MHz (148 SM x 64 lanes), DESIGN.md §4"}
+    aroof, aroof_src = atomic_roof()
+    if aroof:
+        # one fp64 red.add per segment (M7): the tighter of the two roofs
+        kernels["mdnorm"] = {"bound": "atomic", "achieved": stats["segments"] / t / 1e9, "peak": aroof / 1e9,
+                             "unit": "Gatomic/s", "frac": stats["segments"] / t / aroof,
+                             "peak_source": f"measured: {aroof_src} (fp64 red.global.add, L2-resident bins)",
+                             "alu": alu}
+    else:
+        kernels["mdnorm"] = dict(alu, peak_source=f"{peaks_src}: MEASURED_PEAKS.json sm_max_mhz x 148 SM x 64 fp64 lanes")
+    kernels["mdnorm"].update({"kernels": "mdnorm_cull_kernel + mdnorm_walk_kernel", "traffic": md_traffic,
+                              "ms": ph_ms["mdnorm"], "ops_per_launch": md_ops,
+                              "segments_per_launch": stats["segments"]})
     t = ph_ms["binmd"] / 1e3
     bm_bytes = BYTES_PER_EVENT * len(ev)
     kernels["binmd_kernel"] = {"bound": "hbm", "achieved": bm_bytes / t / 1e9, "peak": hbm,
@@ -345,8 +366,7 @@ def run_ours(args, rank, world, local_rank):
     dom = max(("mdnorm", "binmd_kernel"), key=lambda k: kernels[k]["ms"])
     roof = {k: kernels[dom][k] for k in ("bound", "achieved", "peak", "unit", "frac", "traffic")}
     roof["kernel"] = kernels[dom].get("kernels", dom)
-    roof["peak_source"] = (f"{peaks_src}: MEASURED_PEAKS.json sm_max_mhz x 148 SM x 64 fp64 lanes"
-                           if roof["bound"] == "alu" else f"{peaks_src}: MEASURED_PEAKS.json hbm_gbs")
+    roof["peak_source"] = kernels[dom].get("peak_source", f"{peaks_src}: MEASURED_PEAKS.json hbm_gbs")
 
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
