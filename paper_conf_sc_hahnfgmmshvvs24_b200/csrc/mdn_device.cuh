@@ -190,21 +190,20 @@ __device__ __forceinline__ double flux_at(const FluxView& f, double x) {
 
 // ------------------------------------------------------------------------------ M1-M2
 // v = M q (q = z - d precomputed per pixel), clip [k_min, k_max] to the box slab by slab.
-__device__ __forceinline__ bool traj_clip(const GridC& g, const double v[3], double kmin,
-                                          double kmax, double& kin, double& kout) {
+// r[a] = RN(1 / v[a]) for v[a] != 0 (any value for v[a] == 0)
+__device__ __forceinline__ bool traj_clip_r(const GridC& g, const double v[3], const double r[3], double kmin,
+                                            double kmax, double& kin, double& kout) {
   kin = kmin;
   kout = kmax;
 #pragma unroll
   for (int a = 0; a < 3; ++a) {
     double lk, hk;
     if (v[a] > 0.0) {
-      double r = ddiv(1.0, v[a]);
-      lk = dmul(g.lo[a], r);
-      hk = dmul(g.hi[a], r);
+      lk = dmul(g.lo[a], r[a]);
+      hk = dmul(g.hi[a], r[a]);
     } else if (v[a] < 0.0) {
-      double r = ddiv(1.0, v[a]);
-      lk = dmul(g.hi[a], r);
-      hk = dmul(g.lo[a], r);
+      lk = dmul(g.hi[a], r[a]);
+      hk = dmul(g.lo[a], r[a]);
     } else {
       if (g.lo[a] <= 0.0 && 0.0 < g.hi[a]) continue;
       return false;
@@ -213,6 +212,13 @@ __device__ __forceinline__ bool traj_clip(const GridC& g, const double v[3], dou
     if (hk < kout) kout = hk;
   }
   return kin < kout;
+}
+
+__device__ __forceinline__ bool traj_clip(const GridC& g, const double v[3], double kmin,
+                                          double kmax, double& kin, double& kout) {
+  const double r[3] = {v[0] != 0.0 ? ddiv(1.0, v[0]) : 0.0, v[1] != 0.0 ? ddiv(1.0, v[1]) : 0.0,
+                       v[2] != 0.0 ? ddiv(1.0, v[2]) : 0.0};
+  return traj_clip_r(g, v, r, kmin, kmax, kin, kout);
 }
 
 // ------------------------------------------------------------------------------ M3

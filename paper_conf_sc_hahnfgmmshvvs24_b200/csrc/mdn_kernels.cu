@@ -119,10 +119,12 @@ __device__ __forceinline__ void pixel_krange(const MdnParams& p, int64_t pixel, 
 // read once; matrices are warp-uniform smem broadcasts).  A conservative fp32 slab test with a
 // proven error margin rejects most misses without any fp64 division; every
 // survivor gets the exact fp64 v and clip, so the hit decision is the definition's.
+// Rows are stored in test order (fewest bins first: the thin axis of a 2-D slice rejects almost
+// every trajectory after one row product, so the other two rows are only read when a lane of the
+// warp survives it).
 struct alignas(16) CullMat {
-  float M[9];
-  float lot[3], hit[3];  // per-axis fp32 acceptance window [lo - delta, hi + delta)
-  float pad;
+  float4 a[3];  // test-order axis k: (row of fp32(M), acceptance window low lo - delta)
+  float4 hi;    // acceptance window high hi + delta per test-order axis (w unused)
 };
 
 template <bool kStats>
@@ -134,18 +136,24 @@ mdnorm_cull_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ 
   CullMat* sF = reinterpret_cast<CullMat*>(sC + mb.nmat);
   stage_mdnorm_mats(mb, sM, sC);
   __syncthreads();
+  // test order: fewest bins first (stable)
+  int ord[3] = {0, 1, 2};
+  if (p.g.n[ord[1]] < p.g.n[ord[0]]) { const int t = ord[0]; ord[0] = ord[1]; ord[1] = t; }
+  if (p.g.n[ord[2]] < p.g.n[ord[1]]) { const int t = ord[1]; ord[1] = ord[2]; ord[2] = t; }
+  if (p.g.n[ord[1]] < p.g.n[ord[0]]) { const int t = ord[0]; ord[0] = ord[1]; ord[1] = t; }
   for (int m = threadIdx.x; m < mb.nmat; m += blockDim.x) {
-    for (int a = 0; a < 3; ++a) {
-      double sum = 0.0;
-      for (int i = 0; i < 3; ++i) {
-        sF[m].M[3 * a + i] = (float)sM[9 * m + 3 * a + i];
-        sum += fabs(sM[9 * m + 3 * a + i]);
-      }
+    float hi[3];
+#pragma unroll
+    for (int k = 0; k < 3; ++k) {
+      const int a = ord[k];
+      const double* row = sM + 9 * m + 3 * a;
+      const double sum = fabs(row[0]) + fabs(row[1]) + fabs(row[2]);
       // |q_i| <= 2; fp32 v and x = k v are within 1e-6 kmax sum|M_a| of the exact values
       const double delta = 4e-6 * p.kmax * sum + 1e-6 * (fabs(p.g.lo[a]) + fabs(p.g.hi[a])) + 1e-30;
-      sF[m].lot[a] = (float)p.g.lo[a] - (float)delta;
-      sF[m].hit[a] = (float)p.g.hi[a] + (float)delta;
+      sF[m].a[k] = make_float4((float)row[0], (float)row[1], (float)row[2], (float)p.g.lo[a] - (float)delta);
+      hi[k] = (float)p.g.hi[a] + (float)delta;
     }
+    sF[m].hi = make_float4(hi[0], hi[1], hi[2], 0.f);
   }
   __syncthreads();
   const int lane = threadIdx.x & 31;
@@ -175,12 +183,15 @@ mdnorm_cull_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ 
         const double v2 = row_dot(M + 6, px.x, px.y, px.z);
         const double vv[3] = {v0, v1, v2};
         double kin, kout;
+        // one reciprocal per axis serves the clip and the crossing ranges (the same RN(1/v))
+        const double rr[3] = {v0 != 0.0 ? ddiv(1.0, v0) : 0.0, v1 != 0.0 ? ddiv(1.0, v1) : 0.0,
+                              v2 != 0.0 ? ddiv(1.0, v2) : 0.0};
         // a non-finite v (only from a singular composition) contributes nothing in the oracle
-        if (isfinite(v0) && isfinite(v1) && isfinite(v2) && traj_clip(p.g, vv, klo, khi, kin, kout)) {
+        if (isfinite(v0) && isfinite(v1) && isfinite(v2) && traj_clip_r(p.g, vv, rr, klo, khi, kin, kout)) {
           hit = true;
-          const AxisStream s0 = axis_stream(p.g, 0, v0, v0 != 0.0 ? ddiv(1.0, v0) : 0.0, kin, kout);
-          const AxisStream s1 = axis_stream(p.g, 1, v1, v1 != 0.0 ? ddiv(1.0, v1) : 0.0, kin, kout);
-          const AxisStream s2 = axis_stream(p.g, 2, v2, v2 != 0.0 ? ddiv(1.0, v2) : 0.0, kin, kout);
+          const AxisStream s0 = axis_stream(p.g, 0, v0, rr[0], kin, kout);
+          const AxisStream s1 = axis_stream(p.g, 1, v1, rr[1], kin, kout);
+          const AxisStream s2 = axis_stream(p.g, 2, v2, rr[2], kin, kout);
           const int total = s0.cnt + s1.cnt + s2.cnt;
           // piece plan: cut at crossings of the busiest axis A, ~kPieceSegs segments per piece
           const bool a1 = s1.cnt > s0.cnt;
@@ -217,9 +228,14 @@ mdnorm_cull_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ 
     __syncwarp();
   };
 
-  const uint32_t stride = gridDim.x * blockDim.x;
-  // warp-uniform loops so that the ballots below always have the full warp
-  for (uint32_t base = blockIdx.x * blockDim.x + (threadIdx.x & ~31u); base < p.plen; base += stride) {
+  // warps claim 32 pixels at a time from a global cursor (the hit fraction varies strongly over
+  // the detector, so a static split leaves a tail of busy warps); loops are warp-uniform so the
+  // ballots below always have the full warp
+  for (;;) {
+    uint32_t base = 0;
+    if (lane == 0) base = atomicAdd(&p.ctr->pclaim, 32u);
+    base = __shfl_sync(kFull, base, 0);
+    if (base >= p.plen) break;
     const uint32_t off = base + lane;
     const bool valid = off < p.plen;
     double4 px = make_double4(0.0, 0.0, 0.0, 0.0);
@@ -234,24 +250,34 @@ mdnorm_cull_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ 
     const bool live = valid && px.w != 0.0 && klo < khi;
     const float q0 = (float)px.x, q1 = (float)px.y, q2 = (float)px.z;
     const float kmin32 = (float)klo, kmax32 = (float)khi;
+    if (!__any_sync(kFull, live)) continue;
     for (int m = 0; m < mb.nmat; ++m) {
-      const CullMat cm = sF[m];
+      const CullMat* cm = sF + m;
+      const float4 hw = cm->hi;
       bool maybe = live;
-#pragma unroll
-      for (int a = 0; a < 3; ++a) {  // branch-free: all three slabs
-        const float v = fmaf(cm.M[3 * a + 2], q2, fmaf(cm.M[3 * a + 1], q1, cm.M[3 * a] * q0));
+      {  // the most selective axis first
+        const float4 r = cm->a[0];
+        const float v = fmaf(r.z, q2, fmaf(r.y, q1, r.x * q0));
         const float xa = kmin32 * v, xb = kmax32 * v;
-        const float xl = fminf(xa, xb), xh = fmaxf(xa, xb);
-        maybe &= (xh >= cm.lot[a]) & (xl < cm.hit[a]);
+        maybe &= (fmaxf(xa, xb) >= r.w) & (fminf(xa, xb) < hw.x);
       }
-      const unsigned mask = __ballot_sync(kFull, maybe);
-      if (maybe) {
-        const int slot = (qhead + qcnt + __popc(mask & ((1u << lane) - 1u))) & 63;
-        qoff[slot] = off;
-        qmat[slot] = (uint32_t)m;
+      if (__any_sync(kFull, maybe)) {
+#pragma unroll
+        for (int k = 1; k < 3; ++k) {
+          const float4 r = cm->a[k];
+          const float v = fmaf(r.z, q2, fmaf(r.y, q1, r.x * q0));
+          const float xa = kmin32 * v, xb = kmax32 * v;
+          maybe &= (fmaxf(xa, xb) >= r.w) & (fminf(xa, xb) < (k == 1 ? hw.y : hw.z));
+        }
+        const unsigned mask = __ballot_sync(kFull, maybe);
+        if (maybe) {
+          const int slot = (qhead + qcnt + __popc(mask & ((1u << lane) - 1u))) & 63;
+          qoff[slot] = off;
+          qmat[slot] = (uint32_t)m;
+        }
+        qcnt += __popc(mask);
+        if (qcnt >= 32) drain(32);
       }
-      qcnt += __popc(mask);
-      if (qcnt >= 32) drain(32);
     }
   }
   if (qcnt > 0) drain(qcnt);

@@ -49,7 +49,8 @@ struct alignas(16) Hitter {
 struct DevCounters {
   unsigned int nhit;     // hitters written by the cull kernel
   unsigned int claimed;  // hitters claimed by the walk kernel's warps
-  unsigned int pad[2];
+  unsigned int pclaim;   // slab pixels claimed by the cull kernel's warps
+  unsigned int pad;
 };
 
 struct MdnParams {
