@@ -21,11 +21,11 @@ namespace mdn {
 
 namespace {
 
-// One persistent walk CTA per SM (the shared-memory flux table takes up to 180 KB): 896 threads
-// for 2-D slices (measured: 2 x 448 > 2 x 384 ~ 2 x 512 on the CORELLI slab), 768 for 3-D grids
-// (the unrolled walk needs more registers).
+// One persistent walk CTA per SM (the shared-memory flux table takes up to 196 KB): 1024
+// threads for 2-D slices (64 registers: measured 1024 > 896 > 768 on the CORELLI slab), 768 for
+// 3-D grids (the unrolled walk needs more registers).
 #ifndef MDN_WALK_THREADS
-#define MDN_WALK_THREADS 896
+#define MDN_WALK_THREADS 1024
 #endif
 #ifndef MDN_WALK_THREADS_3D
 #define MDN_WALK_THREADS_3D 768
