@@ -27,7 +27,7 @@ def child(args):
     g = m.mdnorm_create_grid(0, wl.lo, wl.hi, wl.nbins, wl.W, m.MDN_ACC_F64)
     m.mdnorm_set_instrument(g, wl.pix_dir, wl.solid)
     m.mdnorm_set_flux(g, wl.flux_k, wl.flux_F)
-    ev = torch.from_numpy(synth.events_for_run(wl, 0)).cuda()
+    ev = torch.from_numpy(synth.events_for_run(wl, 0, order=args.order)).cuda()
     ts = {"mdnorm": [], "binmd": []}
     for it in range(args.iters + 2):
         m.mdnorm_reset(g)
@@ -56,6 +56,7 @@ def main():
     ap.add_argument("--config", default="corelli")
     ap.add_argument("--nops", type=int, default=None)
     ap.add_argument("--events", type=int, default=0)
+    ap.add_argument("--order", default="morton", help="event order: morton | shuffled")
     ap.add_argument("--iters", type=int, default=5)
     ap.add_argument("--libs", default="")
     ap.add_argument("--child", action="store_true")
@@ -68,7 +69,7 @@ def main():
         if lib:
             env["MDN_LIB_PATH"] = os.path.abspath(lib)
         cmd = [sys.executable, __file__, "--child", "--config", args.config, "--iters", str(args.iters),
-               "--events", str(args.events)]
+               "--events", str(args.events), "--order", args.order]
         if args.nops:
             cmd += ["--nops", str(args.nops)]
         r = subprocess.run(cmd, env=env, capture_output=True, text=True)
