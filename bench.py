@@ -385,7 +385,7 @@ def run_ours(args, rank, world, local_rank):
                 "d2h_bytes_per_step": 8 * g.nbins_total,
                 "clocks": clk_e2e.summary(),
                 "path": "C ABI with pinned host events (chunked H2D overlapped with BinMD) and host xs"},
-        "gpu_launches": args.steps * (2 + (1 if rank == 0 else 0)),
+        "gpu_launches": args.steps * (3 + (1 if rank == 0 else 0)),  # cull, walk, binmd (+ xs)
         "roofline": roof,
         "kernels": kernels,
     }

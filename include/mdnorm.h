@@ -146,6 +146,14 @@ mdn_status mdnorm_cross_section(mdn_grid *g, double *xs, void *stream);
  * are both host or both device arrays of nbins_total doubles. */
 mdn_status mdnorm_cross_section_err(mdn_grid *g, double *xs, double *xs_err, void *stream);
 
+/* X2 on a bin shard (after a reduce_scatter of the histograms each GPU divides
+ * its own bins; "the sum of all histograms over the sum of all normalizations", P:72, P:84,
+ * P:100): xs[b] = binmd[b] / norm[b] for b in [0, n), NaN where norm[b] == 0 (reading #12).
+ * norm, binmd and xs are DEVICE arrays of n doubles on `device` (caller-owned; xs may alias
+ * neither input); stream-ordered on `stream`.  MDN_EINVAL for n < 0, NULL or host pointers. */
+mdn_status mdn_divide(int device, const double *norm, const double *binmd, double *xs, int64_t n,
+                      void *stream);
+
 /* Zero all histograms (stream-ordered). */
 mdn_status mdnorm_reset(mdn_grid *g, void *stream);
 

@@ -10,6 +10,6 @@ from .mdnorm import (  # noqa: F401
     mdnorm_cross_section, mdnorm_reset, mdnorm_stats, mdn_last_error, mdn_version,
     mdnorm_set_pixel_krange, mdnorm_set_flux_tables, binmd_accumulate_err, mdnorm_error_histogram, mdnorm_cross_section_err,
     mdnorm_accumulate_matrices, binmd_accumulate_matrices, mdnorm_debug_trajectories,
-    binmd_debug_bins, mdnorm_debug_compose, packed_histograms,
+    binmd_debug_bins, mdnorm_debug_compose, packed_histograms, mdn_divide,
 )
-from .dist import plan_shards, reduce_packed, RankPlan  # noqa: F401
+from .dist import plan_shards, reduce_packed, reduce_scatter_packed, RankPlan  # noqa: F401

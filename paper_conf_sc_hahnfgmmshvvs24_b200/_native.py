@@ -32,6 +32,7 @@ SIGNATURES = {
     "binmd_accumulate": [P, P, i32, P, i64, P, i64, i32, i32, P],
     "mdnorm_histograms": [P, P, P, P],
     "mdnorm_cross_section": [P, P, P],
+    "mdn_divide": [C.c_int, P, P, P, i64, P],
     "mdnorm_reset": [P, P],
     "mdnorm_set_pixel_krange": [P, i64, P, P],
     "mdnorm_set_flux_tables": [P, i32, P, P, P, i64, P],

@@ -756,6 +756,23 @@ mdn_status mdnorm_cross_section_err(mdn_grid* g, double* xs, double* xs_err, voi
   return ok();
 }
 
+mdn_status mdn_divide(int device, const double* norm, const double* binmd, double* xs, int64_t n,
+                      void* stream) {
+  if (n < 0) return fail(MDN_EINVAL, "n < 0");
+  if (n == 0) return ok();
+  if (!norm || !binmd || !xs) return fail(MDN_EINVAL, "NULL argument");
+  int ndev = 0;
+  MDN_CUDA(cudaGetDeviceCount(&ndev), "cudaGetDeviceCount");
+  if (device < 0 || device >= ndev) return fail(MDN_EINVAL, "device %d outside [0, %d)", device, ndev);
+  DeviceGuard dg(device);
+  if (!is_device_ptr(norm) || !is_device_ptr(binmd) || !is_device_ptr(xs))
+    return fail(MDN_EINVAL, "mdn_divide needs device arrays");
+  int nsm = 148;
+  cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, device);
+  MDN_CUDA(mdn::launch_cross_section(norm, binmd, xs, n, nsm, (cudaStream_t)stream), "xs kernel");
+  return ok();
+}
+
 mdn_status mdnorm_cross_section(mdn_grid* g, double* xs, void* stream) {
   if (!g) return fail(MDN_EINVAL, "grid is NULL");
   if (!xs) return fail(MDN_EINVAL, "xs is NULL");

@@ -8,7 +8,9 @@ function is used to add histograms").  Here:
     detector region (balances the CORELLI slab, where only ~4% of trajectories hit the grid),
     and that run's events split into contiguous ranges;
   * exchange      -> ONE collective over the packed fp64 [norm | binmd] buffer (sum); rank 0
-    (or every rank for all_reduce) then divides.
+    (or every rank for all_reduce) then divides -- or, for grids too large to gather on one
+    GPU (the 500^3 stress grid: 2 GB packed), ONE reduce_scatter that leaves every rank the summed
+    norm and binmd of its own contiguous bin block, which it divides locally (mdn_divide).
 The plan is pure Python (tested on CPU with gloo); the reduce works on any torch process group
 (NCCL over NVLink/NVSwitch on B200s).
 """
@@ -72,3 +74,33 @@ def reduce_packed(packed, group=None, dst: int | None = 0):
     if buf is not packed:
         packed.copy_(buf)
     return packed
+
+
+def reduce_scatter_packed(packed, group=None):
+    """Sum the packed [norm | binmd] histograms of all ranks with ONE reduce_scatter; rank r gets
+    bins [b0, b1) (contiguous blocks of ceil(nbins / world)) of both halves.
+
+    Returns (norm_shard, binmd_shard, (b0, b1)) -- views of a new buffer; divide them with
+    mdn_divide.  The bin blocks are laid out rank-major ([rank][norm|binmd][block], zero padded)
+    before the collective so that each rank's output is [norm block | binmd block]."""
+    import torch
+    import torch.distributed as dist
+    n = packed.numel() // 2
+    if not dist.is_available() or not dist.is_initialized() or dist.get_world_size(group) == 1:
+        return packed[:n], packed[n:2 * n], (0, n)
+    world, rank = dist.get_world_size(group), dist.get_rank(group)
+    chunk = -(-n // world)
+    tmp = packed.new_zeros(2, world * chunk)
+    tmp[0, :n] = packed[:n]
+    tmp[1, :n] = packed[n:2 * n]
+    src = tmp.view(2, world, chunk).transpose(0, 1).contiguous().view(-1)  # [rank][half][block]
+    out = packed.new_empty(2 * chunk)
+    if dist.get_backend(group) == "gloo":  # gloo (CPU tests) has no reduce_scatter: all_reduce + slice
+        buf = src.cpu() if src.is_cuda else src
+        dist.all_reduce(buf, op=dist.ReduceOp.SUM, group=group)
+        out.copy_(buf.view(world, 2 * chunk)[rank])
+    else:
+        dist.reduce_scatter_tensor(out, src, op=dist.ReduceOp.SUM, group=group)
+    b0 = min(n, rank * chunk)
+    b1 = min(n, b0 + chunk)
+    return out[: b1 - b0], out[chunk: chunk + b1 - b0], (b0, b1)

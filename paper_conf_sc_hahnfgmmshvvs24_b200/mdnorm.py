@@ -228,6 +228,24 @@ def mdnorm_cross_section(g: Grid, xs=None, stream=None):
     return xs
 
 
+def mdn_divide(norm, binmd, xs=None, stream=None):
+    """X2 on device tensors (a bin shard after a reduce_scatter): xs = binmd / norm, NaN where
+    norm == 0.  norm, binmd (and xs, allocated if None) are contiguous float64 CUDA tensors."""
+    import torch
+    for name, t in (("norm", norm), ("binmd", binmd)):
+        if not (_is_torch(t) and t.is_cuda and t.dtype == torch.float64 and t.is_contiguous()):
+            raise ValueError(f"{name} must be a contiguous float64 CUDA tensor")
+    n = norm.numel()
+    if binmd.numel() != n:
+        raise ValueError("norm and binmd differ in length")
+    if xs is None:
+        xs = torch.empty_like(norm)
+    dev = norm.device.index or 0
+    check(load().mdn_divide(dev, norm.data_ptr(), binmd.data_ptr(), xs.data_ptr(), n, _stream(stream, dev)),
+          "mdn_divide")
+    return xs
+
+
 def mdnorm_reset(g: Grid, stream=None) -> None:
     check(load().mdnorm_reset(g.handle, _stream(stream, g.device)), "mdnorm_reset")
 

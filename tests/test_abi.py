@@ -18,7 +18,7 @@ def lib():
 
 def test_header_symbols_exported(lib):
     names = _native.header_functions()
-    assert len(names) == 23
+    assert len(names) == 24
     for n in names:
         assert hasattr(lib, n), f"{n} declared in include/mdnorm.h but not exported"
         assert n in _native.SIGNATURES, f"{n} missing from the Python binding"
@@ -103,3 +103,11 @@ def test_product_package_never_imports_oracle():
                 src = open(os.path.join(root, f)).read()
                 assert "import oracle" not in src and "from oracle" not in src, f
                 assert "liboracle" not in src and "oracle.h" not in src, f
+
+
+def test_divide_validates_before_cuda(lib):
+    x = np.zeros(4)
+    p = x.ctypes.data
+    assert lib.mdn_divide(0, p, p, p, -1, None) == _native.MDN_EINVAL
+    assert lib.mdn_divide(0, None, p, p, 4, None) == _native.MDN_EINVAL
+    assert lib.mdn_divide(0, p, p, p, 0, None) == _native.MDN_OK  # empty shard: nothing to do

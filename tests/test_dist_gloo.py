@@ -10,7 +10,7 @@ import torch
 import torch.distributed as dist
 import torch.multiprocessing as mp
 
-from paper_conf_sc_hahnfgmmshvvs24_b200.dist import plan_shards, reduce_packed
+from paper_conf_sc_hahnfgmmshvvs24_b200.dist import plan_shards, reduce_packed, reduce_scatter_packed
 
 
 def test_plan_covers_everything_once():
@@ -74,3 +74,49 @@ def test_gloo_world2_reduce_matches_single_process():
         assert p.exitcode == 0
     assert rel_n < 1e-14
     assert abs_b == 0.0  # unit weights: integer counts add exactly
+
+
+def _rs_worker(rank, world, port, out):
+    """reduce_scatter path (SURVEY.md §8(e), 500^3 stress grid): every rank gets the summed norm
+    and binmd of its own bin block; dividing the blocks reproduces the single-process xs."""
+    import oracle
+    import synth
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    wl = synth.make_workload("tiny", events_per_run=3000)
+    wl.nbins = np.array([7, 5, 3])  # 105 bins: not a multiple of the world size (padded blocks)
+    g = oracle.workload_grid(wl)
+    ev = synth.events_for_run(wl, 0)
+    p = plan_shards(world, rank, wl.nruns, wl.npix, len(ev))
+    M = oracle.mdnorm_matrices(wl.R, wl.UB, wl.ops, wl.W)
+    norm = oracle.mdnorm(g, wl.pix_dir, wl.solid, wl.flux_k, wl.flux_F, M, 1.0, wl.k_min, wl.k_max,
+                         pix_begin=p.pix_begin, pix_stride=p.pix_stride)
+    b, e = p.event_ranges[0]
+    bm = oracle.binmd(g, oracle.binmd_matrices(wl.UB, wl.ops, wl.W), ev[b:e])
+    packed = torch.from_numpy(np.concatenate([norm, bm]))
+    ns, bs, (b0, b1) = reduce_scatter_packed(packed)
+    full_n, full_b, full_x = oracle.run_workload(wl, events={0: ev})
+    with np.errstate(invalid="ignore", divide="ignore"):
+        xs = np.where(ns.numpy() > 0, bs.numpy() / ns.numpy(), np.nan)
+    ok = (np.allclose(ns.numpy(), full_n[b0:b1], rtol=1e-14, atol=0) and np.array_equal(bs.numpy(), full_b[b0:b1])
+          and np.array_equal(np.isnan(xs), np.isnan(full_x[b0:b1]))
+          and np.allclose(xs[~np.isnan(xs)], full_x[b0:b1][~np.isnan(xs)], rtol=1e-13))
+    out.put((rank, b0, b1, g.nbins, bool(ok)))
+    dist.destroy_process_group()
+
+
+def test_gloo_world2_reduce_scatter_blocks():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_rs_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    res = sorted(q.get(timeout=300) for _ in range(2))
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert all(r[4] for r in res)
+    # the two blocks tile [0, nbins) exactly
+    assert res[0][1] == 0 and res[0][2] == res[1][1] and res[1][2] == res[0][3]

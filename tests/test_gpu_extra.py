@@ -191,3 +191,37 @@ def test_bench_multi_rank_code_path():
     d = json.loads(lines[0])
     assert d["n_gpus"] == 2 and d["scaling"] == "weak" and d["value"] > 0
     assert d["config"]["trajectories_per_gpu"] == 372736 * 24
+
+
+def test_divide_on_bin_shards(mdn):
+    """X2 per bin block (the reduce_scatter path of SURVEY.md §8(e)): mdn_divide on each block
+    of the summed histograms equals the grid's own cross-section (bit-exact: same IEEE division)
+    and the oracle's xs (NaN masks equal)."""
+    import torch
+    wl = synth.make_workload("tiny")
+    g = mdn.mdnorm_create_grid(0, wl.lo, wl.hi, wl.nbins, wl.W)
+    mdn.mdnorm_set_instrument(g, wl.pix_dir, wl.solid)
+    mdn.mdnorm_set_flux(g, wl.flux_k, wl.flux_F)
+    ev = synth.events_for_run(wl, 0)
+    mdn.mdnorm_accumulate(g, wl.UB, wl.R[0], wl.ops, wl.k_min, wl.k_max, wl.charge[0])
+    mdn.binmd_accumulate(g, wl.UB, wl.ops, torch.from_numpy(ev).cuda())
+    n = g.nbins_total
+    packed = mdn.packed_histograms(g)
+    full = mdn.mdnorm_cross_section(g)
+    world = 3
+    chunk = -(-n // world)
+    parts = []
+    for r in range(world):
+        b0, b1 = min(n, r * chunk), min(n, (r + 1) * chunk)
+        xs = mdn.mdn_divide(packed[b0:b1].contiguous(), packed[n + b0:n + b1].contiguous())
+        parts.append(xs.cpu().numpy())
+    got = np.concatenate(parts)
+    assert np.array_equal(np.isnan(got), np.isnan(full))
+    assert np.array_equal(got[~np.isnan(got)], full[~np.isnan(full)])
+    _, _, oxs = oracle.run_workload(wl, events={0: ev})
+    assert np.array_equal(np.isnan(got), np.isnan(oxs))
+    fin = ~np.isnan(oxs)
+    assert np.all(np.abs(got[fin] - oxs[fin]) <= 3e-12 * np.abs(oxs[fin]))
+    with pytest.raises(ValueError):
+        mdn.mdn_divide(packed[:4].cpu(), packed[:4].cpu())
+    g.close()
