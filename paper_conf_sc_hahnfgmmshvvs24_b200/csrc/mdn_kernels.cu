@@ -200,15 +200,22 @@ mdnorm_cull_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ 
           const AxisStream sa = a2 ? s2 : s01;
           const int A = a2 ? 2 : (a1 ? 1 : 0);
           int P = 1, G = 1;
-          if (total + 1 > kPieceSegs && sa.cnt > 1) {
-            // G crossings of A per piece bring ~G (total + 1) / cA segments: aim at kPieceSegs
-            G = max(1, (kPieceSegs * sa.cnt + (total + 1) / 2) / (total + 1));
+          const int S = p.g.n[2] > 1 ? kPieceSegs3D : kPieceSegs;
+          if (total + 1 > S && sa.cnt > 1) {
+            // G crossings of A per piece bring ~G (total + 1) / cA segments: aim at S
+            G = max(1, (S * sa.cnt + (total + 1) / 2) / (total + 1));
             P = (sa.cnt + G - 1) / G;
           }
           h.v0 = v0; h.v1 = v1; h.v2 = v2; h.kin = kin; h.kout = kout;
           h.oc = dmul(px.w, sC[m]);
           h.A = A | ((p.ptab ? p.ptab[pixel] : 0) << 2);  // busiest axis | flux table << 2
+#if MDN_PIECE_BALANCED
+          // cuts at crossings floor(p cA / P) of axis A (p = 1 .. P-1): the crossings of every axis
+          // are equally spaced in k, so the P pieces get equal segment counts (no short remainder)
+          h.jA = sa.j; h.stepG = sa.step * sa.cnt; h.P = P;
+#else
           h.jA = sa.j; h.stepG = sa.step * G; h.P = P;
+#endif
           if (kStats) {
             c_hit += 1;
             c_cross += total;
@@ -406,8 +413,14 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
       if (h.P > 1) {
         const double vA = A == 0 ? v0 : (A == 1 ? v1 : v2);
         const double rA = ddiv(1.0, vA);
+#if MDN_PIECE_BALANCED
+        const int cA = abs(h.stepG), st = h.stepG < 0 ? -1 : 1;
+        if (mypi > 0) lo_k = plane_k(p.g, A, h.jA + st * ((mypi * cA) / h.P), rA);
+        if (mypi < h.P - 1) hi_k = plane_k(p.g, A, h.jA + st * (((mypi + 1) * cA) / h.P), rA);
+#else
         if (mypi > 0) lo_k = plane_k(p.g, A, h.jA + mypi * h.stepG, rA);
         if (mypi < h.P - 1) hi_k = plane_k(p.g, A, h.jA + (mypi + 1) * h.stepG, rA);
+#endif
       }
       int nc;
       int ns;

@@ -11,10 +11,17 @@ constexpr int kMaxOps = 48;           // MDN_MAX_OPS
 constexpr int kMaxMats = 64;          // MDN_MAX_MATS
 constexpr int kRunsPerLaunch = 16;    // runs composed per MDNorm launch (batched API)
 constexpr int kFluxSmemMax = 4096;    // flux knots staged in shared memory (48 B per knot: 196 KB)
+#ifndef MDN_PIECE_BALANCED
+#define MDN_PIECE_BALANCED 1  // equal-length pieces (cuts at floor(p cA / P)); 0: every G-th crossing
+#endif
 #ifndef MDN_PIECE_SEGS
-#define MDN_PIECE_SEGS 40  // measured: 40 > 24 > 16 (TOPAZ 200^3), ~flat on the CORELLI slab
+#define MDN_PIECE_SEGS 40  // 2-D slices; measured (balanced pieces): 40 > 32 > 48 on the CORELLI slab
+#endif
+#ifndef MDN_PIECE_SEGS_3D
+#define MDN_PIECE_SEGS_3D 56  // 3-D grids; measured (balanced pieces): 56 > 48 > 40 > 32 on TOPAZ 200^3
 #endif
 constexpr int kPieceSegs = MDN_PIECE_SEGS;  // target segments per work piece (load balance, M4-M7)
+constexpr int kPieceSegs3D = MDN_PIECE_SEGS_3D;
 
 // Matrices for one launch, passed by value as a __grid_constant__ kernel parameter (sm_70+
 // kernels accept up to 32 KB of parameters; CUDA >= 12.1).  Either compose (UB, W, ops, R) on
@@ -37,8 +44,10 @@ struct MatBlock {
 };
 
 // A trajectory that hits the grid (output of the cull kernel, input of the walk kernel): its
-// direction v, clip [kin, kout], weight Omega_p c_r, and how it is cut into P pieces at the
-// crossings of axis A with indices j_A + p * stepG (p = 1 .. P-1).
+// direction v, clip [kin, kout], weight Omega_p c_r, and how it is cut into P pieces at
+// crossings of axis A: with MDN_PIECE_BALANCED, stepG = step * cA (signed crossing count of A)
+// and cut p (p = 1 .. P-1) is the crossing with index j_A + step * floor(p cA / P); otherwise
+// the crossing with index j_A + p * stepG.
 struct alignas(16) Hitter {
   double v0, v1, v2, kin;
   double kout, oc;
