@@ -45,9 +45,11 @@
  *  - Precision: geometry (matrices, clip, crossings, midpoints, bin indices, flux
  *    interpolation) is IEEE fp64 without FMA contraction, so crossing counts and bin indices are
  *    bit-identical to the fp64 oracle.  Global histograms are fp64.  mdn_acc selects the
- *    precision of privatised partial sums: MDN_ACC_F64 = fp64 end to end (this build);
- *    MDN_ACC_F32 (fp32 partials folded into the fp64 histogram, BASELINE north_star fp32 mode)
- *    is reserved and currently rejected with MDN_EINVAL.
+ *    precision of the privatised partial sums (mdnorm_set_privatization): MDN_ACC_F64 = fp64
+ *    end to end; MDN_ACC_F32 = fp32 shared-memory partials folded into the fp64 histogram
+ *    (BASELINE north_star fp32 mode: 1e-5 relative per bin).  Launches that accumulate
+ *    straight into the global histogram (grids larger than shared memory) are fp64 in both
+ *    modes.
  */
 #ifndef MDNORM_H
 #define MDNORM_H
@@ -164,6 +166,21 @@ mdn_status mdnorm_reset(mdn_grid *g, void *stream);
  *  plane crossings kept (M3), segments appended (M7), (event, op) pairs (B2),
  *  (event, op) pairs inside the grid (B3)}.  Synchronises the device when out != NULL. */
 mdn_status mdnorm_stats(mdn_grid *g, int enable, int64_t out[6]);
+
+/* Shared-memory privatisation of the histograms (BASELINE north_star "shared-memory privatised
+ * sub-histograms ... falling back to global red.add when the grid exceeds shared memory";
+ * S§2.8 G2/G3).  Each CTA accumulates into its own copy of the grid in shared memory (fp64, or
+ * fp32 with MDN_ACC_F32) and folds it into the global fp64 histogram with one red.add per
+ * touched bin when it finishes.  mode: -1 = auto (default: privatise when the grid fits and the
+ * launch has more work units than the flush touches bins), 0 = never (always global red.add),
+ * 1 = whenever the grid fits.  Grids that do not fit always use global red.add.  Takes effect
+ * for later accumulate calls; no device work.  MDN_EINVAL: NULL grid or mode outside [-1, 1]. */
+mdn_status mdnorm_set_privatization(mdn_grid *g, int32_t mode);
+
+/* Accumulation path taken by the last MDNorm (out[0]) and BinMD (out[1]) launch on this grid:
+ * 0 = global fp64 red.add, 1 = fp64 shared-memory partials, 2 = fp32 shared-memory partials
+ * (tracing and tests; host only, no synchronisation).  MDN_EINVAL: NULL argument. */
+mdn_status mdnorm_accumulation_paths(mdn_grid *g, int32_t out[2]);
 
 /* Message of the last non-OK status on this thread ("" if none).  Never NULL. */
 const char *mdn_last_error(void);

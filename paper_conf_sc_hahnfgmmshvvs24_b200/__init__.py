@@ -4,7 +4,8 @@ The product is the C-ABI library libmdnorm.so (include/mdnorm.h); this package i
 Python binding (same function names) plus the multi-GPU shard plan / reduce (dist.py).
 """
 from .mdnorm import (  # noqa: F401
-    Grid, MdnError, MDN_ACC_F32, MDN_ACC_F64,
+    Grid, MdnError, MDN_ACC_F32, MDN_ACC_F64, MDN_PRIV_AUTO, MDN_PRIV_OFF, MDN_PRIV_ON,
+    mdnorm_set_privatization, mdnorm_accumulation_paths,
     mdnorm_create_grid, mdnorm_destroy, mdnorm_set_instrument, mdnorm_set_flux,
     mdnorm_accumulate, mdnorm_accumulate_runs, binmd_accumulate, mdnorm_histograms,
     mdnorm_cross_section, mdnorm_reset, mdnorm_stats, mdn_last_error, mdn_version,

@@ -16,6 +16,7 @@ HEADER = os.path.join(os.path.dirname(PKG), "include", "mdnorm.h")
 
 MDN_OK, MDN_EINVAL, MDN_ENOMEM, MDN_ECUDA, MDN_ESTATE = 0, 1, 2, 3, 4
 MDN_ACC_F32, MDN_ACC_F64 = 0, 1
+MDN_PRIV_AUTO, MDN_PRIV_OFF, MDN_PRIV_ON = -1, 0, 1
 MDN_MAX_OPS, MDN_MAX_MATS = 48, 64
 STATUS_NAMES = {0: "MDN_OK", 1: "MDN_EINVAL", 2: "MDN_ENOMEM", 3: "MDN_ECUDA", 4: "MDN_ESTATE"}
 
@@ -40,6 +41,8 @@ SIGNATURES = {
     "mdnorm_error_histogram": [P, P],
     "mdnorm_cross_section_err": [P, P, P, P],
     "mdnorm_stats": [P, C.c_int, P],
+    "mdnorm_set_privatization": [P, i32],
+    "mdnorm_accumulation_paths": [P, P],
     "mdn_last_error": [],
     "mdn_version": [],
     "mdnorm_accumulate_matrices": [P, i32, P, P, d, d, i64, i64, i64, P],

@@ -23,6 +23,8 @@ struct mdn_grid {
   GridC g{};
   double W[9]{};
   mdn_acc acc = MDN_ACC_F64;
+  int32_t priv = -1;          // shared-memory privatisation: -1 auto, 0 never, 1 whenever it fits
+  int32_t path[2] = {0, 0};   // accumulation path of the last MDNorm / BinMD launch
   double* d_hist = nullptr;  // [norm | binmd | err2], 3 * nbins doubles
   double2* d_pkr = nullptr;  // per-pixel (k_lo, k_hi) limits, or nullptr
   double4* d_pix = nullptr;
@@ -177,6 +179,7 @@ mdn::MdnParams mdn_params(mdn_grid* g, double k_min, double k_max, int64_t pix_b
   p.fviews = g->nftables > 1 ? g->d_fviews : nullptr;
   p.ptab = g->nftables > 1 ? g->d_ptab : nullptr;
   p.acc_f32 = g->acc == MDN_ACC_F32;
+  p.priv = g->priv;
   p.kmin = k_min;
   p.kmax = k_max;
   p.norm = g->d_hist;
@@ -215,6 +218,7 @@ mdn_status run_mdnorm(mdn_grid* g, mdn::MdnParams p, const MatBlock& mb, cudaStr
     p.p0 = (uint32_t)p0;
     p.plen = (uint32_t)std::min<uint64_t>(per, (uint64_t)p.nshard - p0);
     MDN_CUDA(mdn::launch_mdnorm(p, mb, g->num_sms, s), "mdnorm kernels");
+    g->path[0] = mdn::last_mdnorm_path();
   }
   return MDN_OK;
 }
@@ -251,6 +255,7 @@ mdn::BinParams bin_params(mdn_grid* g, const float* ev, int64_t n, const EvLayou
   std::stable_sort(ord, ord + 3, [&](int a, int b) { return g->g.n[a] < g->g.n[b]; });
   for (int a = 0; a < 3; ++a) p.ord[a] = ord[a];
   p.acc_f32 = g->acc == MDN_ACC_F32;
+  p.priv = g->priv;
   p.binmd = g->d_hist + g->g.nbins;
   p.err2 = g->d_hist + 2 * g->g.nbins;
   p.stats = g->stats_on ? g->d_stats : nullptr;
@@ -297,6 +302,7 @@ mdn_status binmd_host_stream(mdn_grid* g, const MatBlock& mb, int64_t nevents, c
     MDN_CUDA(cudaEventRecord(g->ev_ready[slot], g->copy_stream), "event record");
     MDN_CUDA(cudaStreamWaitEvent(s, g->ev_ready[slot], 0), "wait");
     MDN_CUDA(mdn::launch_binmd(bin_params(g, g->d_stage[slot], n, L), mb, g->num_sms, s), "binmd kernel");
+    g->path[1] = mdn::last_binmd_path();
     MDN_CUDA(cudaEventRecord(g->ev_free[slot], s), "event record");
   }
   return MDN_OK;
@@ -307,6 +313,7 @@ mdn_status binmd_run(mdn_grid* g, const MatBlock& mb, int64_t nevents, const flo
   if (nevents == 0) return ok();
   if (is_device_ptr(events)) {
     MDN_CUDA(mdn::launch_binmd(bin_params(g, events, nevents, L), mb, g->num_sms, s), "binmd kernel");
+    g->path[1] = mdn::last_binmd_path();
     return ok();
   }
   mdn_status st = binmd_host_stream(g, mb, nevents, events, L, s);
@@ -336,7 +343,6 @@ mdn_status mdnorm_create_grid(int device, const double lo[3], const double hi[3]
   }
   if (!finite_all(W, 9) || !nonsingular(W)) return fail(MDN_EINVAL, "W is singular or non-finite");
   if (acc != MDN_ACC_F64 && acc != MDN_ACC_F32) return fail(MDN_EINVAL, "unknown accumulation mode %d", (int)acc);
-  if (acc == MDN_ACC_F32) return fail(MDN_EINVAL, "MDN_ACC_F32 is not available in this build (use MDN_ACC_F64)");
   int ndev = 0;
   cudaError_t e = cudaGetDeviceCount(&ndev);
   if (e != cudaSuccess) return cuda_fail(e, "cudaGetDeviceCount");
@@ -795,6 +801,20 @@ mdn_status mdnorm_reset(mdn_grid* g, void* stream) {
   DeviceGuard dg(g->device);
   MDN_CUDA(cudaMemsetAsync(g->d_hist, 0, sizeof(double) * 3 * g->g.nbins, (cudaStream_t)stream), "memset");
   if (g->d_stats) MDN_CUDA(cudaMemsetAsync(g->d_stats, 0, sizeof(unsigned long long) * 6, (cudaStream_t)stream), "memset");
+  return ok();
+}
+
+mdn_status mdnorm_set_privatization(mdn_grid* g, int32_t mode) {
+  if (!g) return fail(MDN_EINVAL, "grid is NULL");
+  if (mode < -1 || mode > 1) return fail(MDN_EINVAL, "privatization mode must be -1, 0 or 1");
+  g->priv = mode;
+  return ok();
+}
+
+mdn_status mdnorm_accumulation_paths(mdn_grid* g, int32_t out[2]) {
+  if (!g || !out) return fail(MDN_EINVAL, "NULL argument");
+  out[0] = g->path[0];
+  out[1] = g->path[1];
   return ok();
 }
 

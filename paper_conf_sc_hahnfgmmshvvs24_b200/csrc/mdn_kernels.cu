@@ -13,6 +13,7 @@
 //   X2                xs_kernel
 // The parity entry points (debug_*) run the very same device functions (mdn_device.cuh).
 #include <algorithm>
+#include <type_traits>
 
 #include "mdn_kernels.cuh"
 #include "mdn_walk.cuh"
@@ -38,6 +39,10 @@ namespace {
 #define MDN_WALK_CHUNK 8
 #endif
 constexpr int kWalkChunk = MDN_WALK_CHUNK;
+// auto privatisation of the walk: trajectories per (bin x CTA) of the flush (3-D grids; x16 for 2-D)
+#ifndef MDN_PRIV_TRAJ_PER_BIN
+#define MDN_PRIV_TRAJ_PER_BIN 1
+#endif
 constexpr int kWalkRing = 64;  // >= 31 + the largest claim (32), a power of two
 static_assert(kWalkChunk >= 1 && kWalkChunk <= 32, "walk claim size");
 constexpr int kThreads = 256;
@@ -89,6 +94,40 @@ __device__ __forceinline__ void flush_counter(unsigned long long* dst, unsigned 
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) v += __shfl_down_sync(kFull, v, o);
   if ((threadIdx.x & 31) == 0 && v) atomicAdd(dst, v);
+}
+
+// Shared-memory privatised histogram (S§2.8 G2/G3): T = double (MDN_ACC_F64) or float
+// (MDN_ACC_F32 partials); flushed into the fp64 global histogram at the end of the kernel.
+template <typename T>
+struct SmemEmit {
+  T* h;
+  __device__ __forceinline__ void operator()(int b, double val) const { atomicAdd(h + b, (T)val); }
+};
+
+// Zero the CTA's private histogram (before the kernel's first __syncthreads).
+template <typename T>
+__device__ __forceinline__ void priv_zero(T* h, int64_t n) {
+  for (int64_t i = threadIdx.x; i < n; i += blockDim.x) h[i] = T(0);
+}
+
+// Fold the CTA's private histogram into the global fp64 one: one red.add per touched bin
+// (every contribution is >= 0 for MDNorm; a BinMD bin whose weights cancel to 0 is skipped,
+// which leaves the same sum).  Call after a __syncthreads.
+template <typename T>
+__device__ __forceinline__ void priv_flush(const T* h, double* dst, int64_t n) {
+  for (int64_t i = threadIdx.x; i < n; i += blockDim.x) {
+    const T v = h[i];
+    if (v != T(0)) atomicAdd(dst + i, (double)v);
+  }
+}
+
+// kPriv: 0 = global fp64 red.add, 1 = fp64 shared-memory partials, 2 = fp32 shared-memory partials
+template <int kPriv>
+using priv_t = typename std::conditional<kPriv == 2, float, double>::type;
+
+// bytes of a private histogram of n bins, rounded up to 16
+__host__ __device__ constexpr size_t priv_bytes(int kind, int64_t n) {
+  return kind == 0 ? 0 : (((size_t)n * (kind == 2 ? 4 : 8) + 15) & ~(size_t)15);
 }
 
 struct AtomicEmit {
@@ -298,18 +337,22 @@ mdnorm_cull_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ 
 // ---------------------------------------------------------------- M3-M7: balanced piece walk
 // kFlux: 0 = one flux table read from global memory, 1 = one table staged in shared memory,
 // 2 = per-bank tables (pixel -> table map, NEXT #1) read from global memory
-template <int kFlux, bool kStats, bool k3D>
+template <int kFlux, bool kStats, bool k3D, int kPriv>
 __global__ void __launch_bounds__(walk_threads(k3D), MDN_WALK_MINB)
 mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
   constexpr bool kSmemFlux = kFlux == 1;
+  using PT = priv_t<kPriv>;
   extern __shared__ double4 wsm[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int nwarps = blockDim.x >> 5;
-  // shared layout: interval records ka, kb (n double2 each) | knots (n + 2, even) | cell table
-  // (uint16, even) | per-warp prefix sums (32 int) | per-warp hitter rings (kWalkRing unsigned)
+  // shared layout: private histogram (kPriv, 16-byte rounded) | interval records ka, kb (n
+  // double2 each) | knots (n + 2, even) | cell table (uint16, even) | per-warp prefix sums (32
+  // int) | per-warp hitter rings (kWalkRing unsigned)
+  PT* sHist = reinterpret_cast<PT*>(wsm);
+  if (kPriv) priv_zero(sHist, p.g.nbins);
   const int n_rec = kSmemFlux ? p.flux.n : 0;
   const int n_kn = kSmemFlux ? (p.flux.n + 3) & ~1 : 0;
-  double2* sKa = reinterpret_cast<double2*>(wsm);
+  double2* sKa = reinterpret_cast<double2*>(reinterpret_cast<char*>(wsm) + priv_bytes(kPriv, p.g.nbins));
   double2* sKb = sKa + n_rec;
   double* sKn = reinterpret_cast<double*>(sKb + n_rec);
   uint16_t* sTab = reinterpret_cast<uint16_t*>(sKn + n_kn);
@@ -336,7 +379,9 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
     fx.tab = sTab;
   }
   int* pre = sPre + 32 * warp;
-  AtomicEmit emit{p.norm};
+  typename std::conditional<kPriv != 0, SmemEmit<PT>, AtomicEmit>::type emit;
+  if constexpr (kPriv != 0) emit.h = sHist;
+  else emit.h = p.norm;
   const unsigned nhit = *(volatile unsigned*)&p.ctr->nhit;
   unsigned long long c_seg = 0;
   // Per-warp queue of hitters (ring of kWalkRing indices; the head hitter may be partly
@@ -436,6 +481,10 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
     }
     __syncwarp();
   }
+  if (kPriv) {
+    __syncthreads();
+    priv_flush(sHist, p.norm, p.g.nbins);
+  }
   if (kStats) flush_counter(p.stats + 3, c_seg);
 }
 
@@ -453,9 +502,10 @@ struct BinAxis32 {
 // Member loop of one queued (event, class) pair: the remaining two axes of every op of the
 // class, bin and fp64 red.add.  Out of line so that its constants are not hoisted into the
 // class-test loop.  Returns the number of (event, op) pairs that landed inside the grid.
+template <int kPriv>
 __device__ __noinline__ unsigned binmd_members(const BinParams& p, const double* sN, const BinAxis32* sA,
                                                const int* sCls, const int* sMem, float4 ev, float e2, int c,
-                                               int a0, int a1) {
+                                               int a0, int a1, priv_t<kPriv>* hb, priv_t<kPriv>* he) {
   const float w = ev.x, q0 = ev.y, q1 = ev.z, q2 = ev.w;
   const float qm = fmaxf(fabsf(q0), fmaxf(fabsf(q1), fabsf(q2)));
   const int j0 = sCls[c], j1 = sCls[c + 1];
@@ -497,18 +547,37 @@ __device__ __noinline__ unsigned binmd_members(const BinParams& p, const double*
       if (be < 0) continue;
       b = (int)be;
     }
-    atomicAdd(p.binmd + b, (double)w);
-    if (p.col_e >= 0) atomicAdd(p.err2 + b, (double)e2);
+    if constexpr (kPriv != 0) {
+      atomicAdd(hb + b, (priv_t<kPriv>)w);
+      if (p.col_e >= 0) atomicAdd(he + b, (priv_t<kPriv>)e2);
+    } else {
+      atomicAdd(p.binmd + b, (double)w);
+      if (p.col_e >= 0) atomicAdd(p.err2 + b, (double)e2);
+    }
     ++inside;
   }
   return inside;
 }
 
-template <bool kPacked, bool kStats>
-__global__ void __launch_bounds__(kThreads)
+// Block size: 256 threads with global reductions (several CTAs per SM); 512 with a private
+// shared-memory histogram (fewer, larger CTAs: the histogram is zeroed and flushed per CTA).
+__host__ __device__ constexpr int bin_threads(int kPriv) { return kPriv ? 512 : kThreads; }
+
+template <bool kPacked, bool kStats, int kPriv>
+__global__ void __launch_bounds__(bin_threads(kPriv), kPriv ? 2 : 4)
 binmd_kernel(const __grid_constant__ BinParams p, const __grid_constant__ MatBlock mb) {
+  constexpr int kBT = bin_threads(kPriv);
+  using PT = priv_t<kPriv>;
   __shared__ double sN[kMaxMats * 9];
   __shared__ BinAxis32 sA[kMaxMats * 3];
+  // private histograms (kPriv): binmd, then err2 when the error column is read
+  extern __shared__ double4 bsm[];
+  PT* hb = reinterpret_cast<PT*>(bsm);
+  PT* he = reinterpret_cast<PT*>(reinterpret_cast<char*>(bsm) + priv_bytes(kPriv, p.g.nbins));
+  if (kPriv) {
+    priv_zero(hb, p.g.nbins);
+    if (p.col_e >= 0) priv_zero(he, p.g.nbins);
+  }
   stage_binmd_mats(mb, sN);
   __syncthreads();
   for (int i = threadIdx.x; i < 3 * mb.nmat; i += blockDim.x) {
@@ -566,9 +635,9 @@ binmd_kernel(const __grid_constant__ BinParams p, const __grid_constant__ MatBlo
   const int lane = threadIdx.x & 31;
   // per-warp queue of (event, class) pairs that pass the class test: their member loop runs
   // only when 32 are queued, with the warp converged
-  __shared__ float4 sQv[(kThreads / 32) * 64];
-  __shared__ int sQc[(kThreads / 32) * 64];
-  __shared__ float sQe[(kThreads / 32) * 64];  // error-squared column (col_e >= 0 only)
+  __shared__ float4 sQv[(kBT / 32) * 64];
+  __shared__ int sQc[(kBT / 32) * 64];
+  __shared__ float sQe[(kBT / 32) * 64];  // error-squared column (col_e >= 0 only)
   float4* qv = sQv + (threadIdx.x >> 5) * 64;
   int* qc = sQc + (threadIdx.x >> 5) * 64;
   float* qe = sQe + (threadIdx.x >> 5) * 64;
@@ -581,7 +650,8 @@ binmd_kernel(const __grid_constant__ BinParams p, const __grid_constant__ MatBlo
     __syncwarp();
     if (lane < n) {
       const int slot = (qhead + lane) & 63;
-      c_in += binmd_members(p, sN, sA, sCls, sMem, qv[slot], has_err ? qe[slot] : 0.0f, qc[slot], a0, a1);
+      c_in += binmd_members<kPriv>(p, sN, sA, sCls, sMem, qv[slot], has_err ? qe[slot] : 0.0f, qc[slot], a0,
+                                   a1, hb, he);
     }
     qhead = (qhead + n) & 63;
     qcnt -= n;
@@ -658,6 +728,11 @@ binmd_kernel(const __grid_constant__ BinParams p, const __grid_constant__ MatBlo
     cur_e = nxt_e;
   }
   if (qcnt > 0) drain(qcnt);
+  if (kPriv) {
+    __syncthreads();
+    priv_flush(hb, p.binmd, p.g.nbins);
+    if (p.col_e >= 0) priv_flush(he, p.err2, p.g.nbins);
+  }
   if (kStats) {
     flush_counter(p.stats + 4, c_pairs);
     flush_counter(p.stats + 5, c_in);
@@ -784,11 +859,11 @@ size_t walk_smem(const MdnParams& p, bool smem_flux, int threads) {
          (sizeof(int) * 32 + 2 * sizeof(unsigned) * kWalkRing) * (threads / 32);
 }
 
-template <int kFlux, bool kStats, bool k3D>
+template <int kFlux, bool kStats, bool k3D, int kPriv>
 cudaError_t launch_walk(const MdnParams& p, int num_sms, cudaStream_t s) {
   constexpr int threads = walk_threads(k3D);
-  const size_t smem = walk_smem(p, kFlux == 1, threads);
-  auto k = mdnorm_walk_kernel<kFlux, kStats, k3D>;
+  const size_t smem = walk_smem(p, kFlux == 1, threads) + priv_bytes(kPriv, p.g.nbins);
+  auto k = mdnorm_walk_kernel<kFlux, kStats, k3D, kPriv>;
   cudaError_t err = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (err != cudaSuccess) return err;
   int per_sm = 0;
@@ -796,6 +871,24 @@ cudaError_t launch_walk(const MdnParams& p, int num_sms, cudaStream_t s) {
   if (err != cudaSuccess) return err;
   k<<<num_sms * std::max(per_sm, 1), threads, smem, s>>>(p);
   return cudaGetLastError();
+}
+
+template <int kFlux, int kPriv>
+cudaError_t launch_walk_d(const MdnParams& p, bool d3, int num_sms, cudaStream_t s) {
+  if (d3) return p.stats ? launch_walk<kFlux, true, true, kPriv>(p, num_sms, s)
+                         : launch_walk<kFlux, false, true, kPriv>(p, num_sms, s);
+  return p.stats ? launch_walk<kFlux, true, false, kPriv>(p, num_sms, s)
+                 : launch_walk<kFlux, false, false, kPriv>(p, num_sms, s);
+}
+
+thread_local int g_last_mdnorm_path = 0;
+thread_local int g_last_binmd_path = 0;
+
+int smem_optin(cudaError_t* err) {
+  int dev = 0, smem_max = 0;
+  if ((*err = cudaGetDevice(&dev)) != cudaSuccess) return 0;
+  *err = cudaDeviceGetAttribute(&smem_max, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+  return smem_max;
 }
 
 template <bool kStats>
@@ -813,14 +906,26 @@ cudaError_t launch_cull(const MdnParams& p, const MatBlock& mb, int num_sms, cud
   return cudaGetLastError();
 }
 
-template <bool kPacked, bool kStats>
-cudaError_t launch_binmd_t(const BinParams& p, const MatBlock& mb, int num_sms, cudaStream_t s) {
-  auto k = binmd_kernel<kPacked, kStats>;
-  int per_sm = 0;
-  cudaError_t err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kThreads, 0);
+template <bool kPacked, bool kStats, int kPriv>
+cudaError_t launch_binmd_t(const BinParams& p, const MatBlock& mb, int num_sms, size_t smem, cudaStream_t s) {
+  constexpr int threads = bin_threads(kPriv);
+  auto k = binmd_kernel<kPacked, kStats, kPriv>;
+  cudaError_t err = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (err != cudaSuccess) return err;
-  k<<<grid_for(p.nevents, num_sms, std::max(per_sm, 1)), kThreads, 0, s>>>(p, mb);
+  int per_sm = 0;
+  err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, threads, smem);
+  if (err != cudaSuccess) return err;
+  k<<<grid_for(p.nevents, num_sms, std::max(per_sm, 1), threads), threads, smem, s>>>(p, mb);
   return cudaGetLastError();
+}
+
+template <int kPriv>
+cudaError_t launch_binmd_p(const BinParams& p, const MatBlock& mb, bool packed, int num_sms, size_t smem,
+                           cudaStream_t s) {
+  if (packed) return p.stats ? launch_binmd_t<true, true, kPriv>(p, mb, num_sms, smem, s)
+                             : launch_binmd_t<true, false, kPriv>(p, mb, num_sms, smem, s);
+  return p.stats ? launch_binmd_t<false, true, kPriv>(p, mb, num_sms, smem, s)
+                 : launch_binmd_t<false, false, kPriv>(p, mb, num_sms, smem, s);
 }
 
 }  // namespace
@@ -839,29 +944,77 @@ cudaError_t launch_mdnorm(const MdnParams& p, const MatBlock& mb, int num_sms, c
   if (err != cudaSuccess) return err;
   // 2-D slices (a single bin on the last axis, "lBins=1") merge two crossing streams
   const bool d3 = p.g.n[2] > 1;
+  const int smem_max = smem_optin(&err);
+  if (err != cudaSuccess) return err;
+  const int threads = walk_threads(d3);
   // the flux table goes to shared memory when it fits one CTA (uint16 cell entries)
-  int dev = 0, smem_max = 0;
-  if ((err = cudaGetDevice(&dev)) != cudaSuccess) return err;
-  if ((err = cudaDeviceGetAttribute(&smem_max, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev)) != cudaSuccess)
-    return err;
-  const bool fits = p.flux.n <= kFluxSmemMax && walk_smem(p, true, walk_threads(d3)) <= (size_t)smem_max;
-  const int mode = p.fviews ? 2 : (fits ? 1 : 0);
-#define MDN_WALK_DISPATCH(F)                                                                    \
-  if (d3) return p.stats ? launch_walk<F, true, true>(p, num_sms, s) : launch_walk<F, false, true>(p, num_sms, s); \
-  return p.stats ? launch_walk<F, true, false>(p, num_sms, s) : launch_walk<F, false, false>(p, num_sms, s);
-  if (mode == 1) { MDN_WALK_DISPATCH(1) }
-  if (mode == 2) { MDN_WALK_DISPATCH(2) }
-  MDN_WALK_DISPATCH(0)
-#undef MDN_WALK_DISPATCH
+  const bool flux_fits = p.flux.n <= kFluxSmemMax && walk_smem(p, true, threads) <= (size_t)smem_max;
+  // Private shared-memory histogram (S§2.8 G2) when the grid fits next to the walk's other shared
+  // data: with the flux table in shared memory if both fit, else with the flux read through L1.
+  // priv = 1 takes it whenever it fits; auto (-1) when the launch's trajectories outnumber the
+  // bins the flush touches (one CTA per SM flushes every bin) by MDN_PRIV_TRAJ_PER_BIN (3-D
+  // grids: every trajectory crosses the box) or 16x that (2-D slices: a few % hit the slab).
+  // Measured (tools/priv_sweep.sh): TOPAZ 8 ops on 16^3 - 25^3 grids 2.1-3.2x faster; CORELLI
+  // 24 ops on 16^2 / 60^2 slabs 2.7x / 1.2x faster, on 100^2 equal, on 150^2 1.35x slower.
+  const int kind = p.acc_f32 ? 2 : 1;
+  const size_t hb = priv_bytes(kind, p.g.nbins);
+  const bool priv_ok = p.priv != 0 && !p.fviews;
+  const uint64_t per_bin = (uint64_t)MDN_PRIV_TRAJ_PER_BIN * (d3 ? 1u : 16u);
+  const bool worth = p.priv == 1 ||
+                     (uint64_t)p.plen * (uint64_t)mb.nmat >= (uint64_t)p.g.nbins * (uint64_t)num_sms * per_bin;
+  const bool with_sflux = priv_ok && worth && flux_fits && walk_smem(p, true, threads) + hb <= (size_t)smem_max;
+  const bool with_gflux = priv_ok && worth && !with_sflux && walk_smem(p, false, threads) + hb <= (size_t)smem_max;
+  if (with_sflux || with_gflux) {
+    g_last_mdnorm_path = kind;
+    if (with_sflux) return kind == 2 ? launch_walk_d<1, 2>(p, d3, num_sms, s) : launch_walk_d<1, 1>(p, d3, num_sms, s);
+    return kind == 2 ? launch_walk_d<0, 2>(p, d3, num_sms, s) : launch_walk_d<0, 1>(p, d3, num_sms, s);
+  }
+  g_last_mdnorm_path = 0;
+  if (p.fviews) return launch_walk_d<2, 0>(p, d3, num_sms, s);
+  if (flux_fits) return launch_walk_d<1, 0>(p, d3, num_sms, s);
+  return launch_walk_d<0, 0>(p, d3, num_sms, s);
 }
 
 cudaError_t launch_binmd(const BinParams& p, const MatBlock& mb, int num_sms, cudaStream_t s) {
   if (p.nevents <= 0 || mb.nmat <= 0) return cudaSuccess;
   const bool packed = p.stride == 4 && p.col_w == 0 && p.col_q == 1 &&
                       (reinterpret_cast<uintptr_t>(p.events) & 15) == 0;
-  if (packed) return p.stats ? launch_binmd_t<true, true>(p, mb, num_sms, s) : launch_binmd_t<true, false>(p, mb, num_sms, s);
-  return p.stats ? launch_binmd_t<false, true>(p, mb, num_sms, s) : launch_binmd_t<false, false>(p, mb, num_sms, s);
+  // Private shared-memory histogram(s) (S§2.8 G3) when binmd (+ err2) fit one 512-thread CTA
+  // next to its static shared data.  priv = 1 takes it whenever it fits; auto (-1) only when two
+  // CTAs fit per SM (with one, 16 warps per SM cannot keep the event stream going) and the
+  // (event, op) pairs outnumber the flushed bins by 64 (measured, tools/priv_sweep.sh: TOPAZ
+  // 8 ops on 16^3 / 20^3 2.5x faster, CORELLI 24 ops on 16^2 2.6x and 60^2 1.1x faster; a
+  // 100^2 slab, one CTA per SM, 1.5x slower).
+  cudaError_t err = cudaSuccess;
+  const int smem_max = smem_optin(&err);
+  if (err != cudaSuccess) return err;
+  const int kind = p.acc_f32 ? 2 : 1;
+  const size_t hb = priv_bytes(kind, p.g.nbins) * (p.col_e >= 0 ? 2 : 1);
+  if (p.priv != 0) {
+    cudaFuncAttributes fa{};
+    err = packed ? cudaFuncGetAttributes(&fa, binmd_kernel<true, false, 1>)
+                 : cudaFuncGetAttributes(&fa, binmd_kernel<false, false, 1>);
+    if (err != cudaSuccess) return err;
+    int dev = 0, sm_smem = 0;
+    if ((err = cudaGetDevice(&dev)) != cudaSuccess) return err;
+    if ((err = cudaDeviceGetAttribute(&sm_smem, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev)) != cudaSuccess)
+      return err;
+    const size_t per_cta = fa.sharedSizeBytes + hb + 1024;  // + the per-CTA reservation
+    const bool fits = per_cta <= (size_t)smem_max;
+    const uint64_t ctas = (uint64_t)num_sms * 2;
+    const bool worth = p.priv == 1 || (2 * per_cta <= (size_t)sm_smem &&
+                                       (uint64_t)p.nevents * (uint64_t)mb.nmat >= (uint64_t)p.g.nbins * ctas * 64);
+    if (fits && worth) {
+      g_last_binmd_path = kind;
+      return kind == 2 ? launch_binmd_p<2>(p, mb, packed, num_sms, hb, s) : launch_binmd_p<1>(p, mb, packed, num_sms, hb, s);
+    }
+  }
+  g_last_binmd_path = 0;
+  return launch_binmd_p<0>(p, mb, packed, num_sms, 0, s);
 }
+
+int last_mdnorm_path() { return g_last_mdnorm_path; }
+int last_binmd_path() { return g_last_binmd_path; }
 
 cudaError_t launch_cross_section(const double* norm, const double* binmd, double* xs, int64_t nbins,
                                  int num_sms, cudaStream_t s) {

@@ -70,7 +70,8 @@ struct MdnParams {
   FluxView flux;           // table 0 (device pointers, global)
   const FluxView* fviews;  // per-bank tables (several tables), or nullptr
   const int32_t* ptab;     // pixel -> flux table (with fviews), or nullptr
-  int32_t acc_f32;
+  int32_t acc_f32;         // privatised partial sums in fp32 (MDN_ACC_F32) instead of fp64
+  int32_t priv;            // shared-memory privatised histogram: -1 auto, 0 never, 1 whenever it fits
   double kmin, kmax;
   double* norm;            // fp64 histogram (nbins)
   unsigned long long* stats;  // nullptr, or [traj, hits, crossings, segments] (+= per launch)
@@ -87,7 +88,8 @@ struct BinParams {
   int32_t col_w, col_q;
   int32_t col_e;           // error-squared column, or -1
   int32_t ord[3];          // axis test order of the fp32 fast path (fewest bins first)
-  int32_t acc_f32;
+  int32_t acc_f32;         // privatised partial sums in fp32 (MDN_ACC_F32) instead of fp64
+  int32_t priv;            // shared-memory privatised histogram: -1 auto, 0 never, 1 whenever it fits
   double* binmd;           // fp64 histogram (nbins)
   double* err2;            // fp64 error-squared histogram (nbins), used when col_e >= 0
   unsigned long long* stats;  // nullptr, or [.., .., .., .., pairs, inside] (+= per launch)
@@ -99,6 +101,10 @@ cudaError_t launch_pixels_prepare(const double* dir, const double* solid, double
 // MDNorm for shard pixels [p.p0, p.p0 + p.plen) x all matrices: cull (M1-M3) + piece walk (M3-M7).
 cudaError_t launch_mdnorm(const MdnParams& p, const MatBlock& mb, int num_sms, cudaStream_t s);
 cudaError_t launch_binmd(const BinParams& p, const MatBlock& mb, int num_sms, cudaStream_t s);
+// Accumulation path chosen for the last launch_mdnorm / launch_binmd on this thread (tracing and
+// tests): 0 = global fp64 red.add, 1 = shared-memory fp64 partials, 2 = shared-memory fp32 partials.
+int last_mdnorm_path();
+int last_binmd_path();
 cudaError_t launch_cross_section(const double* norm, const double* binmd, double* xs, int64_t nbins,
                                  int num_sms, cudaStream_t s);
 cudaError_t launch_cross_section_err(const double* norm, const double* binmd, const double* err2, double* xs,

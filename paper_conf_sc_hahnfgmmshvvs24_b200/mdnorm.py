@@ -10,7 +10,8 @@ import ctypes as C
 import numpy as np
 
 from . import _native
-from ._native import MDN_ACC_F32, MDN_ACC_F64, MdnError, check, load  # noqa: F401
+from ._native import (MDN_ACC_F32, MDN_ACC_F64, MDN_PRIV_AUTO, MDN_PRIV_OFF, MDN_PRIV_ON,  # noqa: F401
+                      MdnError, check, load)
 
 
 def _is_torch(x) -> bool:
@@ -259,6 +260,21 @@ def mdnorm_stats(g: Grid, enable: int = -1, read: bool = True):
     out = np.zeros(6, np.int64)
     check(load().mdnorm_stats(g.handle, int(enable), out.ctypes.data if read else None), "mdnorm_stats")
     return dict(zip(STAT_NAMES, (int(x) for x in out))) if read else None
+
+
+def mdnorm_set_privatization(g: Grid, mode: int) -> None:
+    """Shared-memory privatised histograms: MDN_PRIV_AUTO (-1), MDN_PRIV_OFF (0), MDN_PRIV_ON (1)."""
+    check(load().mdnorm_set_privatization(g.handle, int(mode)), "mdnorm_set_privatization")
+
+
+PATH_NAMES = {0: "global", 1: "smem_f64", 2: "smem_f32"}
+
+
+def mdnorm_accumulation_paths(g: Grid) -> tuple[str, str]:
+    """Accumulation path of the last (MDNorm, BinMD) launch: 'global', 'smem_f64' or 'smem_f32'."""
+    out = np.zeros(2, np.int32)
+    check(load().mdnorm_accumulation_paths(g.handle, out.ctypes.data), "mdnorm_accumulation_paths")
+    return PATH_NAMES[int(out[0])], PATH_NAMES[int(out[1])]
 
 
 def mdn_last_error() -> str:

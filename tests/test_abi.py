@@ -18,7 +18,7 @@ def lib():
 
 def test_header_symbols_exported(lib):
     names = _native.header_functions()
-    assert len(names) == 24
+    assert len(names) == 26
     for n in names:
         assert hasattr(lib, n), f"{n} declared in include/mdnorm.h but not exported"
         assert n in _native.SIGNATURES, f"{n} missing from the Python binding"
@@ -77,6 +77,8 @@ def test_null_handles_are_einval(lib):
     assert lib.mdnorm_cross_section(None, z.ctypes.data, None) == _native.MDN_EINVAL
     assert lib.mdnorm_reset(None, None) == _native.MDN_EINVAL
     assert lib.mdnorm_destroy(None) == _native.MDN_OK
+    assert lib.mdnorm_set_privatization(None, 0) == _native.MDN_EINVAL
+    assert lib.mdnorm_accumulation_paths(None, np.zeros(2, np.int32).ctypes.data) == _native.MDN_EINVAL
 
 
 def test_no_gpu_is_reported_not_crashing(lib):

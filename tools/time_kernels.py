@@ -24,7 +24,9 @@ def child(args):
     import paper_conf_sc_hahnfgmmshvvs24_b200 as m
     wl = synth.make_workload(args.config, nops=args.nops,
                              events_per_run=args.events if args.events else None)
-    g = m.mdnorm_create_grid(0, wl.lo, wl.hi, wl.nbins, wl.W, m.MDN_ACC_F64)
+    nbins = [int(x) for x in args.nbins.split("x")] if args.nbins else wl.nbins
+    g = m.mdnorm_create_grid(0, wl.lo, wl.hi, nbins, wl.W, args.acc)
+    m.mdnorm_set_privatization(g, args.priv)
     m.mdnorm_set_instrument(g, wl.pix_dir, wl.solid)
     m.mdnorm_set_flux(g, wl.flux_k, wl.flux_F)
     ev = torch.from_numpy(synth.events_for_run(wl, 0, order=args.order)).cuda()
@@ -47,6 +49,7 @@ def child(args):
     st = m.mdnorm_stats(g, 0)
     out = {k: float(np.mean(v)) for k, v in ts.items()}
     out["segments"] = st["segments"]
+    out["paths"] = m.mdnorm_accumulation_paths(g)
     out["norm_sum"] = float(m.packed_histograms(g)[: g.nbins_total].sum().item())
     print(json.dumps(out))
 
@@ -59,6 +62,9 @@ def main():
     ap.add_argument("--order", default="morton", help="event order: morton | shuffled")
     ap.add_argument("--iters", type=int, default=5)
     ap.add_argument("--libs", default="")
+    ap.add_argument("--nbins", default="", help="override the grid, e.g. 60x60x1")
+    ap.add_argument("--priv", type=int, default=-1, help="privatisation: -1 auto, 0 off, 1 on")
+    ap.add_argument("--acc", type=int, default=1, help="1 = MDN_ACC_F64, 0 = MDN_ACC_F32")
     ap.add_argument("--child", action="store_true")
     args = ap.parse_args()
     if args.child:
@@ -69,7 +75,10 @@ def main():
         if lib:
             env["MDN_LIB_PATH"] = os.path.abspath(lib)
         cmd = [sys.executable, __file__, "--child", "--config", args.config, "--iters", str(args.iters),
-               "--events", str(args.events), "--order", args.order]
+               "--events", str(args.events), "--order", args.order, "--priv", str(args.priv),
+               "--acc", str(args.acc)]
+        if args.nbins:
+            cmd += ["--nbins", args.nbins]
         if args.nops:
             cmd += ["--nops", str(args.nops)]
         r = subprocess.run(cmd, env=env, capture_output=True, text=True)
