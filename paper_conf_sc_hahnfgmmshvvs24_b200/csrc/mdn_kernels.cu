@@ -39,6 +39,19 @@ namespace {
 #define MDN_WALK_CHUNK 8
 #endif
 constexpr int kWalkChunk = MDN_WALK_CHUNK;
+// claimed hitters sorted by piece length before they enter the warp's queue
+#ifndef MDN_WALK_SORT
+#define MDN_WALK_SORT 1
+#endif
+#ifndef MDN_BINMD_WAGG
+#define MDN_BINMD_WAGG 0  // warp-aggregated BinMD reductions (measured 1.3-1.9x slower: off)
+#endif
+#ifndef MDN_WALK_WAGG
+#define MDN_WALK_WAGG 0  // warp-aggregated walk reductions (measured 1.4-1.75x slower: off)
+#endif
+#ifndef MDN_BINMD_MINB
+#define MDN_BINMD_MINB 4  // resident 256-thread CTAs per SM (caps registers at 64)
+#endif
 // auto privatisation of the walk: trajectories per (bin x CTA) of the flush (3-D grids; x16 for 2-D)
 #ifndef MDN_PRIV_TRAJ_PER_BIN
 #define MDN_PRIV_TRAJ_PER_BIN 1
@@ -96,12 +109,47 @@ __device__ __forceinline__ void flush_counter(unsigned long long* dst, unsigned 
   if ((threadIdx.x & 31) == 0 && v) atomicAdd(dst, v);
 }
 
+// h[b] += v (and h2[b] += v2 when two); with kAgg warp-aggregated: the converged lanes that add
+// to the same bin (events of one Bragg peak arrive together in the MDBox/Morton order) are
+// summed with shuffles and their lowest lane makes the single reduction (S§2.8 G3; north_star
+// "warp-aggregated atomics").  Only the order of the additions changes.  Measured on this B200
+// (DESIGN.md §9): __match_any_sync + the shuffles cost more than the same-address reductions
+// they save -- BinMD 2x slower on the Morton-ordered CORELLI events, 1.8x on TOPAZ 48 ops, 1.6x
+// into a private shared-memory grid; the walk 1.4-1.75x -- so both switches are off.
+template <bool kAgg, typename T>
+__device__ __forceinline__ void agg_add(T* h, T* h2, int b, T v, T v2, bool two) {
+  if constexpr (kAgg) {
+    const unsigned act = __activemask();
+    const unsigned peers = __match_any_sync(act, b);
+    const int lane = threadIdx.x & 31;
+    const int most = (int)__reduce_max_sync(act, (unsigned)__popc(peers));
+    if (most > 1) {
+      unsigned rest = peers & ~(1u << lane);  // the other lanes of this lane's bin
+      for (int r = 1; r < most; ++r) {
+        const int src = rest ? __ffs(rest) - 1 : lane;
+        const T o = __shfl_sync(act, v, src);
+        const T o2 = two ? __shfl_sync(act, v2, src) : T(0);
+        if (rest) {
+          v += o;
+          v2 += o2;
+          rest &= rest - 1u;
+        }
+      }
+    }
+    if (lane != __ffs(peers) - 1) return;
+  }
+  atomicAdd(h + b, v);
+  if (two) atomicAdd(h2 + b, v2);
+}
+
 // Shared-memory privatised histogram (S§2.8 G2/G3): T = double (MDN_ACC_F64) or float
 // (MDN_ACC_F32 partials); flushed into the fp64 global histogram at the end of the kernel.
 template <typename T>
 struct SmemEmit {
   T* h;
-  __device__ __forceinline__ void operator()(int b, double val) const { atomicAdd(h + b, (T)val); }
+  __device__ __forceinline__ void operator()(int b, double val) const {
+    agg_add<MDN_WALK_WAGG != 0, T>(h, nullptr, b, (T)val, T(0), false);
+  }
 };
 
 // Zero the CTA's private histogram (before the kernel's first __syncthreads).
@@ -137,7 +185,9 @@ struct AtomicEmit {
     if (val == -1.2345e300) h[b] = val;
   }
 #else
-  __device__ __forceinline__ void operator()(int b, double val) const { atomicAdd(h + b, val); }
+  __device__ __forceinline__ void operator()(int b, double val) const {
+    agg_add<MDN_WALK_WAGG != 0, double>(h, nullptr, b, val, 0.0, false);
+  }
 #endif
 };
 
@@ -247,7 +297,9 @@ mdnorm_cull_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ 
           }
           h.v0 = v0; h.v1 = v1; h.v2 = v2; h.kin = kin; h.kout = kout;
           h.oc = dmul(px.w, sC[m]);
-          h.A = A | ((p.ptab ? p.ptab[pixel] : 0) << 2);  // busiest axis | flux table << 2
+          // busiest axis | flux table << 2 | min(segments per piece, 1023) << 22 (walk sort key)
+          const int plen = min((total + P) / P, 1023);
+          h.A = A | ((p.ptab ? p.ptab[pixel] : 0) << 2) | (plen << 22);
 #if MDN_PIECE_BALANCED
           // cuts at crossings floor(p cA / P) of axis A (p = 1 .. P-1): the crossings of every axis
           // are equally spaced in k, so the P pieces get equal segment counts (no short remainder)
@@ -411,11 +463,41 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
       // small ones so that the warps finish together
       chunk = nhit - b > tail ? 32u : (unsigned)kWalkChunk;
       int P = 0;
+#if MDN_WALK_SORT
+      // Claimed hitters enter the queue longest pieces first (warp bitonic sort on the piece
+      // length the cull stored), so that a round's 32 pieces have similar lengths and its lanes
+      // finish together.  Key = length << 5 | lane: unique, invalid lanes (0) last.
+      int A = 0;
+      if ((unsigned)lane < nnew) {
+        const int4 t = *reinterpret_cast<const int4*>(&p.hit[b + lane].A);  // (A, jA, stepG, P)
+        A = t.x;
+        P = t.w;
+      }
+      unsigned key = (unsigned)lane < nnew ? ((((unsigned)A >> 22) + 1u) << 5) | (unsigned)lane : 0u;
+#pragma unroll
+      for (int k = 2; k <= 32; k <<= 1) {
+#pragma unroll
+        for (int j = k >> 1; j > 0; j >>= 1) {
+          const unsigned o = __shfl_xor_sync(kFull, key, j);
+          const bool desc = (lane & k) == 0 || k == 32;  // final merge: descending
+          const bool low = (lane & j) == 0;
+          key = (low == desc) ? max(key, o) : min(key, o);
+        }
+      }
+      const int src = key & 31;
+      P = __shfl_sync(kFull, P, src);
+      if ((unsigned)lane >= nnew) P = 0;
+      if ((unsigned)lane < nnew) {
+        ring[(head + nq + lane) & (kWalkRing - 1)] = b + src;
+        ringP[(head + nq + lane) & (kWalkRing - 1)] = P;
+      }
+#else
       if ((unsigned)lane < nnew) {
         P = p.hit[b + lane].P;
         ring[(head + nq + lane) & (kWalkRing - 1)] = b + lane;
         ringP[(head + nq + lane) & (kWalkRing - 1)] = P;
       }
+#endif
       nq += nnew;
       qpieces += __reduce_add_sync(kFull, P);
       __syncwarp();
@@ -472,7 +554,7 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
       if (kFlux == 1) {
         ns = traj_walk<k3D, uint16_t>(p.g, fx, v0, v1, v2, lo_k, hi_k, h.oc, emit, &nc);
       } else if (kFlux == 2) {
-        const FluxView fv = p.fviews[h.A >> 2];
+        const FluxView fv = p.fviews[(h.A >> 2) & 0xFFFFF];
         ns = traj_walk<k3D, int>(p.g, fv, v0, v1, v2, lo_k, hi_k, h.oc, emit, &nc);
       } else {
         ns = traj_walk<k3D, int>(p.g, fx, v0, v1, v2, lo_k, hi_k, h.oc, emit, &nc);
@@ -548,11 +630,9 @@ __device__ __noinline__ unsigned binmd_members(const BinParams& p, const double*
       b = (int)be;
     }
     if constexpr (kPriv != 0) {
-      atomicAdd(hb + b, (priv_t<kPriv>)w);
-      if (p.col_e >= 0) atomicAdd(he + b, (priv_t<kPriv>)e2);
+      agg_add<MDN_BINMD_WAGG != 0>(hb, he, b, (priv_t<kPriv>)w, (priv_t<kPriv>)e2, p.col_e >= 0);
     } else {
-      atomicAdd(p.binmd + b, (double)w);
-      if (p.col_e >= 0) atomicAdd(p.err2 + b, (double)e2);
+      agg_add<MDN_BINMD_WAGG != 0>(p.binmd, p.err2, b, (double)w, (double)e2, p.col_e >= 0);
     }
     ++inside;
   }
@@ -564,7 +644,7 @@ __device__ __noinline__ unsigned binmd_members(const BinParams& p, const double*
 __host__ __device__ constexpr int bin_threads(int kPriv) { return kPriv ? 512 : kThreads; }
 
 template <bool kPacked, bool kStats, int kPriv>
-__global__ void __launch_bounds__(bin_threads(kPriv), kPriv ? 2 : 4)
+__global__ void __launch_bounds__(bin_threads(kPriv), kPriv ? 2 : MDN_BINMD_MINB)
 binmd_kernel(const __grid_constant__ BinParams p, const __grid_constant__ MatBlock mb) {
   constexpr int kBT = bin_threads(kPriv);
   using PT = priv_t<kPriv>;
