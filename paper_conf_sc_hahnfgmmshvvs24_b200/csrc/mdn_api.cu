@@ -480,12 +480,13 @@ mdn_status build_flux_table(const double* hk, const double* hF, int64_t n, HostF
     t.ka[i] = make_double2(hk[i], hF[i]);
     t.kb[i] = make_double2(dF, 1.0 / dk);
   }
-  // cells narrower than 3 x the smallest knot spacing hold at most 3 knots (all fast); four cells
-  // per knot make a knot at or below x in x's own cell rare (the one-probe look-up)
+  t.ka[n - 1] = make_double2(hk[n - 1], hF[n - 1]);  // kappa_{n-1} for probes (MDN_FLUX_NOKN)
+  // cells narrower than 3 x the smallest knot spacing hold at most 3 knots (all fast); eight cells
+  // per knot (MDN_FLUX_CELLS) make a knot at or below x in x's own cell rare (one-probe look-up)
   double hmin = HUGE_VAL;
   for (int64_t i = 0; i + 1 < n; ++i) hmin = std::min(hmin, hk[i + 1] - hk[i]);
   const double want = std::ceil((hk[n - 1] - hk[0]) / (2.9 * hmin));
-  const int ntab = (int)std::min<double>(std::max<double>(4.0 * (double)n, want), (double)(1 << 22));
+  const int ntab = (int)std::min<double>(std::max<double>((double)MDN_FLUX_CELLS * (double)n, want), (double)(1 << 22));
   t.inv_cell = (double)ntab / (hk[n - 1] - hk[0]);
   if (!std::isfinite(t.inv_cell)) return fail(MDN_EINVAL, "flux table k range too small");
   std::vector<double> U((size_t)n);

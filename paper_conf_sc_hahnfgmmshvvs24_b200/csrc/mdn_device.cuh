@@ -116,15 +116,24 @@ __device__ __forceinline__ bool compose_binmd(const double* UB, const double* S,
 // so with s_c = max{i : U_i < c}, i is s_c plus the number of knots of cell c that are <= x:
 // probe kappa_{s_c+1}, kappa_{s_c+2}, ... until the first knot > x (which is kappa_{i+1}, the
 // knot dk_i needs).  The common case -- no knot of cell c at or below x -- needs one probe, and
-// the interval records are loaded alongside it; cells are four per knot (or narrower), so a
-// probe finds a knot <= x for ~1/8 of the look-ups.  Cells with more than three knots (and c =
-// 0, x outside the table, or c + 1 > U_{n-1}) are flagged and take the general path: clamps and
-// a bisection.  Two (+inf) pad knots keep the probes in bounds.
+// the interval records are loaded alongside it; cells are MDN_FLUX_CELLS (8) per knot (or
+// narrower), so a probe finds a knot <= x for a small fraction of the look-ups.  Cells with more
+// than three knots (and c = 0, x outside the table, or c + 1 > U_{n-1}) are flagged and take the
+// general path: clamps and a bisection.  A fast cell lies below U_{n-1}, so its probes stop at
+// kappa_{n-1} at the latest: they read kappa_{i+1} from the next interval record (ka[n-1] holds
+// kappa_{n-1}), and the shared-memory copy needs no separate knot array (MDN_FLUX_NOKN; the
+// freed 32 KB pay for the 8 cells per knot: measured 1-2% faster walk than 4 cells + knots).
+// The general path bisects the global knot array (two +inf pads).
 //
-// Shared-memory layout (bank conflicts of random look-ups, measured: profiles/): knots as a
-// dense double array (8-byte probes over 16 bank pairs) and the two records as separate
+// Shared-memory layout (bank conflicts of random look-ups, measured: profiles/): the two records as separate
 // 16-byte-strided double2 arrays (all 8 sixteen-byte bank groups), instead of one 32-byte record
 // per interval (which uses only 4 of the 8 groups).
+#ifndef MDN_FLUX_NOKN
+#define MDN_FLUX_NOKN 1  // no shared-memory knot array: probes read the next interval record (frees 32 KB)
+#endif
+#ifndef MDN_FLUX_CELLS
+#define MDN_FLUX_CELLS 8  // cell-table cells per knot (at least); measured 8 > 6 > 4 with MDN_FLUX_NOKN
+#endif
 constexpr unsigned kFluxDense32 = 1u << 30;  // flag bit in an int32 table entry
 constexpr unsigned kFluxDense16 = 1u << 15;  // flag bit in a uint16 (shared-memory) entry
 
@@ -175,12 +184,22 @@ __device__ __forceinline__ double flux_at(const FluxView& f, double x) {
   const unsigned e = (unsigned)c < (unsigned)f.ntab ? tab_entry<TabT>(f, c) : flag;
   if (e & flag) return flux_general(f, x);
   int i = (int)e;
+  // kappa_{i+1}: from the knot array, or (MDN_FLUX_NOKN) from the next interval record -- the
+  // fast path never looks past kappa_{n-1} (its cells end below U_{n-1})
+#if MDN_FLUX_NOKN
+  double kn1 = f.ka[i + 1].x;
+#else
   double kn1 = f.kn[i + 1];
+#endif
   double2 a = f.ka[i], b = f.kb[i];
   if (kn1 <= x) {  // a knot of cell c lies at or below x (at most three)
     do {
       ++i;
+#if MDN_FLUX_NOKN
+      kn1 = f.ka[i + 1].x;
+#else
       kn1 = f.kn[i + 1];
+#endif
     } while (kn1 <= x);
     a = f.ka[i];
     b = f.kb[i];

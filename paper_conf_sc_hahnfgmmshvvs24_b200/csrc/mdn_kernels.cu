@@ -403,7 +403,7 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
   PT* sHist = reinterpret_cast<PT*>(wsm);
   if (kPriv) priv_zero(sHist, p.g.nbins);
   const int n_rec = kSmemFlux ? p.flux.n : 0;
-  const int n_kn = kSmemFlux ? (p.flux.n + 3) & ~1 : 0;
+  const int n_kn = kSmemFlux && !MDN_FLUX_NOKN ? (p.flux.n + 3) & ~1 : 0;
   double2* sKa = reinterpret_cast<double2*>(reinterpret_cast<char*>(wsm) + priv_bytes(kPriv, p.g.nbins));
   double2* sKb = sKa + n_rec;
   double* sKn = reinterpret_cast<double*>(sKb + n_rec);
@@ -415,7 +415,8 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
       sKa[i] = p.flux.ka[i];
       sKb[i] = p.flux.kb[i];
     }
-    for (int i = threadIdx.x; i < p.flux.n + 2; i += blockDim.x) sKn[i] = p.flux.kn[i];
+    if (!MDN_FLUX_NOKN)
+      for (int i = threadIdx.x; i < p.flux.n + 2; i += blockDim.x) sKn[i] = p.flux.kn[i];
     const int* gtab = static_cast<const int*>(p.flux.tab);
     for (int i = threadIdx.x; i < p.flux.ntab; i += blockDim.x) {
       const unsigned e = (unsigned)gtab[i];
@@ -425,7 +426,7 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
   __syncthreads();
   FluxView fx = p.flux;
   if (kSmemFlux) {
-    fx.kn = sKn;
+    if (!MDN_FLUX_NOKN) fx.kn = sKn;  // else the rare general path bisects the global knots
     fx.ka = sKa;
     fx.kb = sKb;
     fx.tab = sTab;
@@ -933,7 +934,7 @@ int grid_for(int64_t work, int num_sms, int per_sm, int threads = kThreads) {
 
 // dynamic shared memory of the walk kernel (layout in mdnorm_walk_kernel)
 size_t walk_smem(const MdnParams& p, bool smem_flux, int threads) {
-  return (smem_flux ? 2 * sizeof(double2) * p.flux.n + sizeof(double) * ((p.flux.n + 3) & ~1) +
+  return (smem_flux ? 2 * sizeof(double2) * p.flux.n + (MDN_FLUX_NOKN ? 0 : sizeof(double) * ((p.flux.n + 3) & ~1)) +
                           sizeof(uint16_t) * ((p.flux.ntab + 1) & ~1)
                     : 0) +
          (sizeof(int) * 32 + 2 * sizeof(unsigned) * kWalkRing) * (threads / 32);

@@ -10,7 +10,7 @@ namespace mdn {
 constexpr int kMaxOps = 48;           // MDN_MAX_OPS
 constexpr int kMaxMats = 64;          // MDN_MAX_MATS
 constexpr int kRunsPerLaunch = 16;    // runs composed per MDNorm launch (batched API)
-constexpr int kFluxSmemMax = 4096;    // flux knots staged in shared memory (48 B per knot: 196 KB)
+constexpr int kFluxSmemMax = 4096;    // flux knots staged in shared memory (32 B records + 8 x 2 B cells per knot: 192 KB)
 #ifndef MDN_PIECE_BALANCED
 #define MDN_PIECE_BALANCED 1  // equal-length pieces (cuts at floor(p cA / P)); 0: every G-th crossing
 #endif
