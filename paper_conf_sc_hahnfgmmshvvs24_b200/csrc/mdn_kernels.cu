@@ -49,6 +49,9 @@ constexpr int kWalkChunk = MDN_WALK_CHUNK;
 #ifndef MDN_WALK_WAGG
 #define MDN_WALK_WAGG 0  // warp-aggregated walk reductions (measured 1.4-1.75x slower: off)
 #endif
+#ifndef MDN_BINMD_CT
+#define MDN_BINMD_CT 1  // class test rows gathered per class (BinMD -3%)
+#endif
 #ifndef MDN_BINMD_MINB
 #define MDN_BINMD_MINB 4  // resident 256-thread CTAs per SM (caps registers at 64)
 #endif
@@ -712,6 +715,13 @@ binmd_kernel(const __grid_constant__ BinParams p, const __grid_constant__ MatBlo
   }
   __syncthreads();
   const int ncls = sNcls;
+#if MDN_BINMD_CT
+  // class test rows gathered by class index (one level of shared-memory indirection less in the
+  // per-event class loop)
+  __shared__ BinAxis32 sCT[kMaxMats];
+  for (int c = threadIdx.x; c < ncls; c += blockDim.x) sCT[c] = sA[3 * sMem[sCls[c]]];
+  __syncthreads();
+#endif
   const int a0 = p.ord[0], a1 = p.ord[1], a2 = p.ord[2];
   const int lane = threadIdx.x & 31;
   // per-warp queue of (event, class) pairs that pass the class test: their member loop runs
@@ -755,15 +765,9 @@ binmd_kernel(const __grid_constant__ BinParams p, const __grid_constant__ MatBlo
     cur = load(base + lane);
     cur_e = load_e(base + lane);
   }
-  for (; base < p.nevents; base += stride) {
-    const bool valid = base + lane < p.nevents;
-    float4 nxt = make_float4(0.f, 0.f, 0.f, 0.f);  // software prefetch of the next event
-    float nxt_e = 0.f;
-    if (base + stride + lane < p.nevents) {
-      nxt = load(base + stride + lane);
-      nxt_e = load_e(base + stride + lane);
-    }
-    const float q0 = cur.y, q1 = cur.z, q2 = cur.w;
+  // the class tests of one event (per-warp queue of passing (event, class) pairs)
+  auto test_event = [&](const float4 ev, const float ev_e, const bool valid) {
+    const float q0 = ev.y, q1 = ev.z, q2 = ev.w;
     const float qm = fmaxf(fabsf(q0), fmaxf(fabsf(q1), fabsf(q2)));
     if (kStats && valid) c_pairs += mb.nmat;
 #ifdef MDN_BINMD_BOX
@@ -779,7 +783,11 @@ binmd_kernel(const __grid_constant__ BinParams p, const __grid_constant__ MatBlo
 #endif
     for (int c = 0; c < ncls; ++c) {
       // first-tested axis, once for the whole class
+#if MDN_BINMD_CT
+      const BinAxis32 ax = sCT[c];
+#else
       const BinAxis32 ax = sA[3 * sMem[sCls[c]]];
+#endif
 #ifdef MDN_BINMD_BOX
       {  // warp-uniform box test
         const float p0a = ax.r0 * b0l, p0b = ax.r0 * b0h, p1a = ax.r1 * b1l, p1b = ax.r1 * b1h;
@@ -798,13 +806,22 @@ binmd_kernel(const __grid_constant__ BinParams p, const __grid_constant__ MatBlo
       const unsigned mask = __ballot_sync(kFull, pass);
       if (pass) {
         const int slot = (qhead + qcnt + __popc(mask & ((1u << lane) - 1u))) & 63;
-        qv[slot] = cur;
+        qv[slot] = ev;
         qc[slot] = c;
-        if (has_err) qe[slot] = cur_e;
+        if (has_err) qe[slot] = ev_e;
       }
       qcnt += __popc(mask);
       if (qcnt >= 32) drain(32);
     }
+  };
+  for (; base < p.nevents; base += stride) {
+    float4 nxt = make_float4(0.f, 0.f, 0.f, 0.f);  // software prefetch of the next event
+    float nxt_e = 0.f;
+    if (base + stride + lane < p.nevents) {
+      nxt = load(base + stride + lane);
+      nxt_e = load_e(base + stride + lane);
+    }
+    test_event(cur, cur_e, base + lane < p.nevents);
     cur = nxt;
     cur_e = nxt_e;
   }
