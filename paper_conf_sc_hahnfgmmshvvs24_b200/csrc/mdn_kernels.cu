@@ -220,7 +220,7 @@ struct alignas(16) CullMat {
 };
 
 template <bool kStats>
-__global__ void __launch_bounds__(kThreads)
+__global__ void __launch_bounds__(kThreads, 4)  // 64 registers: four resident CTAs per SM
 mdnorm_cull_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ MatBlock mb) {
   extern __shared__ double smem[];
   double* sM = smem;
