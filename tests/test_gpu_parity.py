@@ -103,7 +103,7 @@ def _traj_check(mdn, g, wl, M, charge, ids, orc_grid, max_segs=1024):
     return nc, ns
 
 
-@pytest.mark.parametrize("cfg", ["tiny", "corelli", "topaz"])
+@pytest.mark.parametrize("cfg", ["tiny", "corelli", "topaz", "stress"])
 def test_debug_trajectories_bit_exact(mdn, cfg):
     wl = synth.make_workload(cfg)
     g = make_grid(mdn, wl)
@@ -270,6 +270,31 @@ def test_topaz_full_size_properties(mdn):
     mdn.binmd_accumulate(g, wl.UB, wl.ops, dev_events(events))
     _, bm = hist(mdn, g)
     obm = oracle.binmd(oracle.workload_grid(wl), oracle.binmd_matrices(wl.UB, wl.ops, wl.W), events)
+    assert_rel(bm, obm, what="binmd")
+
+
+# ----------------------------------------------------------------------------- stress (configs[4])
+
+
+def test_stress_500_cubed(mdn):
+    """BASELINE configs[4] grid (500^3 = 1.25e8 bins, 1 GB fp64 histograms: the global-reduction
+    path) with 48 ops, in the bench's launch configuration: every 4099th pixel through the
+    production kernels against the oracle per bin, and 10^6 of its events through BinMD."""
+    wl = synth.make_workload("stress", events_per_run=1_000_000)
+    g = make_grid(mdn, wl)
+    stride = 4099
+    mdn.mdnorm_accumulate(g, wl.UB, wl.R[0], wl.ops, wl.k_min, wl.k_max, 1.0, pix_stride=stride)
+    ev = synth.events_for_run(wl, 0)
+    mdn.binmd_accumulate(g, wl.UB, wl.ops, dev_events(ev))
+    assert mdn.mdnorm_accumulation_paths(g) == ("global", "global")
+    norm, bm = hist(mdn, g)
+    og = oracle.workload_grid(wl)
+    M = oracle.mdnorm_matrices(wl.R, wl.UB, wl.ops, wl.W)
+    onorm = oracle.mdnorm(og, wl.pix_dir, wl.solid, wl.flux_k, wl.flux_F, M, 1.0, wl.k_min, wl.k_max,
+                          pix_stride=stride)
+    assert_rel(norm, onorm, what="norm")
+    del onorm, norm
+    obm = oracle.binmd(og, oracle.binmd_matrices(wl.UB, wl.ops, wl.W), ev)
     assert_rel(bm, obm, what="binmd")
 
 
