@@ -175,40 +175,103 @@ def run_reference(args, rank, world):
     wl = make_bench_workload(1)
     ev = synth.events_for_run(wl, 0)
     stride = args.ref_stride
+    threads = host_threads()
     times = []
     for k in range(args.warmup + args.steps):
-        t = {}
-        t0 = time.perf_counter()
-        oracle.run_workload(wl, events={0: ev}, pix_stride=stride, event_stride=stride, timings=t)
-        dt = time.perf_counter() - t0
+        t_md, t_bm, _, _ = oracle_timed(wl, ev, stride, threads)
         if k >= args.warmup:
-            times.append(t["mdnorm_s"] + t["binmd_s"])
+            times.append(t_md + t_bm)
     traj = wl.npix * wl.nops / stride
     value = traj / statistics.mean(times)
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * statistics.mean(times),
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
             "data": "synthetic (seeded, SURVEY.md §8(d) recipe)", "config": config_dict(wl, 1),
-            "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle",
                              "sample": f"every {stride}th pixel (all 24 ops) and every {stride}th event "
-                                       f"of the CORELLI-shaped run per step; single-threaded C oracle"},
+                                       f"of the CORELLI-shaped run per step; the C oracle on {threads} host "
+                                       f"threads ({host_cpu()}), private histograms per thread"},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
     return 0
 
 
-def cpu_baseline(wl, ev, stride):
+def host_cpu() -> str:
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+def oracle_timed(wl, ev, stride, threads):
+    """The oracle as it stands on every stride-th pixel (all ops) and every stride-th event of run 0,
+    on `threads` host threads: each thread calls the unchanged C oracle (ctypes releases the GIL)
+    on an interleaved pixel shard and a contiguous event shard with its own histograms, summed in
+    fixed order afterwards (S§8(d): "OpenMP over (r, s, pixel-chunk) and (s, event-chunk), with
+    per-thread private fp64 histograms reduced in fixed thread order").  Returns (seconds of
+    MDNorm, seconds of BinMD, norm, binmd)."""
+    from concurrent.futures import ThreadPoolExecutor
+
     import oracle
     oracle.build()
-    t = {}
-    oracle.run_workload(wl, runs=[0], events={0: ev}, pix_stride=stride, event_stride=stride, timings=t)
-    secs = t["mdnorm_s"] + t["binmd_s"]
+    g = oracle.workload_grid(wl)
+    M = oracle.mdnorm_matrices(wl.R[:1], wl.UB, wl.ops, wl.W)
+    N = oracle.binmd_matrices(wl.UB, wl.ops, wl.W)
+    evs = np.ascontiguousarray(ev[::stride])
+    cuts = np.linspace(0, len(evs), threads + 1).astype(np.int64)
+    shards = [np.ascontiguousarray(evs[cuts[t]:cuts[t + 1]]) for t in range(threads)]
+
+    def md(t):
+        a = oracle.Accumulator(g.nbins)
+        oracle.mdnorm(g, wl.pix_dir, wl.solid, wl.flux_k, wl.flux_F, M, wl.charge[0], wl.k_min, wl.k_max,
+                      pix_begin=t * stride, pix_stride=stride * threads, acc=a)
+        return a
+
+    def bm(t):
+        a = oracle.Accumulator(g.nbins)
+        oracle.binmd(g, N, shards[t], acc=a)
+        return a
+
+    with ThreadPoolExecutor(threads) as ex:
+        t0 = time.perf_counter()
+        na = list(ex.map(md, range(threads)))
+        t1 = time.perf_counter()
+        ba = list(ex.map(bm, range(threads)))
+        t2 = time.perf_counter()
+    norm = na[0].value()
+    for a in na[1:]:
+        norm = norm + a.value()
+    bmh = ba[0].value()
+    for a in ba[1:]:
+        bmh = bmh + a.value()
+    return t1 - t0, t2 - t1, norm, bmh
+
+
+def host_threads() -> int:
+    try:
+        return max(1, len(os.sched_getaffinity(0)))
+    except AttributeError:  # pragma: no cover
+        return max(1, os.cpu_count() or 1)
+
+
+def cpu_baseline(wl, ev, stride):
+    threads = host_threads()
+    t_md, t_bm, _, _ = oracle_timed(wl, ev, stride, threads)
+    secs = t_md + t_bm
     traj = wl.npix * wl.nops / stride
-    return {"value": traj / secs, "unit": UNIT, "cores": 1, "kind": "oracle",
+    # single-thread figure on an 8x smaller sample of the same run
+    s1_md, s1_bm, _, _ = oracle_timed(wl, ev, 8 * stride, 1)
+    return {"value": traj / secs, "unit": UNIT, "cores": threads, "kind": "oracle",
             "sample": f"every {stride}th pixel (all {wl.nops} ops) + every {stride}th event of run 0 "
                       f"({traj:.0f} trajectories, {len(ev) // stride} events; "
-                      f"MDNorm {t['mdnorm_s']:.2f} s + BinMD {t['binmd_s']:.2f} s), single thread",
-            "events_per_s": (len(ev) / stride) / secs}
+                      f"MDNorm {t_md:.2f} s + BinMD {t_bm:.2f} s) on {threads} host threads "
+                      f"({host_cpu()}), private histograms per thread",
+            "events_per_s": (len(ev) / stride) / secs,
+            "single_thread": {"value": (traj / 8) / (s1_md + s1_bm), "unit": UNIT,
+                              "sample": f"every {8 * stride}th pixel and event, 1 thread"}}
 
 
 # ----------------------------------------------------------------------------- our arm
@@ -407,8 +470,8 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--cpu-stride", type=int, default=2, help="oracle sample: every n-th pixel and event")
-    ap.add_argument("--ref-stride", type=int, default=8, help="--impl reference per-step sample stride")
+    ap.add_argument("--cpu-stride", type=int, default=1, help="oracle sample: every n-th pixel and event")
+    ap.add_argument("--ref-stride", type=int, default=1, help="--impl reference per-step sample stride")
     ap.add_argument("--json-out", default=None)
     ap.add_argument("--dist-backend", default="nccl",
                     help="nccl (production); gloo + MDN_BENCH_SHARED_GPU=1 exercises the N>1 code "
