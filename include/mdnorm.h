@@ -156,7 +156,9 @@ mdn_status mdnorm_cross_section_err(mdn_grid *g, double *xs, double *xs_err, voi
 mdn_status mdn_divide(int device, const double *norm, const double *binmd, double *xs, int64_t n,
                       void *stream);
 
-/* Zero all histograms (stream-ordered). */
+/* Zero all histograms (stream-ordered) and start an accumulation epoch: host events passed to
+ * later binmd_accumulate* calls are copied to the device only after the stream reaches this
+ * point (the copies still overlap the MDNorm kernels enqueued after it). */
 mdn_status mdnorm_reset(mdn_grid *g, void *stream);
 
 /* Work counters (tracing).  enable = 1 turns counting on for later kernels, 0 turns it off,

@@ -47,6 +47,7 @@ struct mdn_grid {
   cudaStream_t copy_stream = nullptr;
   cudaEvent_t ev_ready[2] = {nullptr, nullptr};
   cudaEvent_t ev_free[2] = {nullptr, nullptr};
+  cudaEvent_t ev_epoch = nullptr;  // recorded by mdnorm_reset: host-event copies start after it
 };
 
 namespace {
@@ -292,6 +293,10 @@ mdn_status binmd_host_stream(mdn_grid* g, const MatBlock& mb, int64_t nevents, c
   // after every scatter launch (never-recorded events are complete).  Nothing else orders the
   // copies after earlier work on the caller's stream, so the first chunks' H2D overlaps the
   // MDNorm kernels enqueued before this call.
+  // The copies are ordered after the caller's last mdnorm_reset (the start of an accumulation
+  // epoch), not after its MDNorm kernels, so they overlap MDNorm without starting before the
+  // epoch the events belong to.
+  if (g->ev_epoch) MDN_CUDA(cudaStreamWaitEvent(g->copy_stream, g->ev_epoch, 0), "wait");
   int64_t c = 0;
   for (int64_t off = 0; off < nevents; off += chunk, ++c) {
     const int slot = (int)(c & 1);
@@ -393,6 +398,7 @@ mdn_status mdnorm_destroy(mdn_grid* g) {
     if (g->ev_ready[i]) cudaEventDestroy(g->ev_ready[i]);
     if (g->ev_free[i]) cudaEventDestroy(g->ev_free[i]);
   }
+  if (g->ev_epoch) cudaEventDestroy(g->ev_epoch);
   if (g->copy_stream) cudaStreamDestroy(g->copy_stream);
   delete g;
   cudaGetLastError();
@@ -802,6 +808,8 @@ mdn_status mdnorm_reset(mdn_grid* g, void* stream) {
   DeviceGuard dg(g->device);
   MDN_CUDA(cudaMemsetAsync(g->d_hist, 0, sizeof(double) * 3 * g->g.nbins, (cudaStream_t)stream), "memset");
   if (g->d_stats) MDN_CUDA(cudaMemsetAsync(g->d_stats, 0, sizeof(unsigned long long) * 6, (cudaStream_t)stream), "memset");
+  if (!g->ev_epoch) MDN_CUDA(cudaEventCreateWithFlags(&g->ev_epoch, cudaEventDisableTiming), "event");
+  MDN_CUDA(cudaEventRecord(g->ev_epoch, (cudaStream_t)stream), "event record");
   return ok();
 }
 
