@@ -12,12 +12,17 @@
 //                        the access pattern of a trajectory's consecutive segments)
 //   red_f32_random  S    the same with fp32
 //   red_shared_f64       fp64 atomicAdd to shared memory (privatised accumulation)
+//   red_shared_f32       fp32 atomicAdd to shared memory (MDN_ACC_F32 partials)
+//   red_dsmem_f64        fp64 atomicAdd to random bins of a histogram distributed over the shared
+//                        memory of an 8-CTA cluster (red.shared::cluster via map_shared_rank)
 //   fp64_alu             independent DADD/DMUL chains (FP64-pipe rate, no FMA)
 // Histogram sizes: CORELLI 600x600 (2.88 MB), TOPAZ 200^3 (64 MB), stress 500^3 (1 GB).
 #include <cstdio>
 #include <cstdint>
 #include <cstdlib>
+#include <cooperative_groups.h>
 #include <cuda_runtime.h>
+namespace cg = cooperative_groups;
 
 #define CK(x)                                                                         \
   do {                                                                                \
@@ -70,6 +75,37 @@ __global__ void red_shared(double* out, int iters, uint32_t nbins) {
   xs32(s);
   for (int i = 0; i < iters; ++i) atomicAdd(sh + below(xs32(s), nbins), 1.0);
   __syncthreads();
+  if (threadIdx.x == 0) out[blockIdx.x] = sh[0];
+}
+
+template <typename T>
+__global__ void red_shared_t(double* out, int iters, uint32_t nbins) {
+  extern __shared__ double shd[];
+  T* sh = reinterpret_cast<T*>(shd);
+  for (uint32_t i = threadIdx.x; i < nbins; i += blockDim.x) sh[i] = T(0);
+  __syncthreads();
+  uint32_t s = 0x51ed27u ^ (blockIdx.x * blockDim.x + threadIdx.x) * 0x85ebca6bu;
+  xs32(s);
+  for (int i = 0; i < iters; ++i) atomicAdd(sh + below(xs32(s), nbins), T(1));
+  __syncthreads();
+  if (threadIdx.x == 0) out[blockIdx.x] = (double)sh[0];
+}
+
+// nbins per CTA; every update goes to a random CTA of the cluster (7/8 of them remote)
+__global__ void red_dsmem(double* out, int iters, uint32_t nbins) {
+  extern __shared__ double sh[];
+  cg::cluster_group cl = cg::this_cluster();
+  for (uint32_t i = threadIdx.x; i < nbins; i += blockDim.x) sh[i] = 0.0;
+  cl.sync();
+  const uint32_t nr = cl.num_blocks();
+  uint32_t s = 0x2545f491u ^ (blockIdx.x * blockDim.x + threadIdx.x) * 0x9e3779b9u;
+  xs32(s);
+  for (int i = 0; i < iters; ++i) {
+    const uint32_t r = xs32(s);
+    double* dst = cl.map_shared_rank(sh, below(r, nr));
+    atomicAdd(dst + below(xs32(s), nbins), 1.0);
+  }
+  cl.sync();
   if (threadIdx.x == 0) out[blockIdx.x] = sh[0];
 }
 
@@ -159,6 +195,26 @@ int main() {
     const float ms = t.best([&] { red_shared<<<blocks, threads, sb * 8>>>(out, it, sb); });
     CK(cudaGetLastError());
     printf(" \"red_shared_f64_per_s\": %.4g,\n", nthr * it / (ms * 1e-3));
+    CK(cudaFuncSetAttribute(red_shared_t<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, sb * 8));
+    const float msf = t.best([&] { red_shared_t<float><<<blocks, threads, sb * 8>>>(out, it, sb); });
+    CK(cudaGetLastError());
+    printf(" \"red_shared_f32_per_s\": %.4g,\n", nthr * it / (msf * 1e-3));
+    // cluster of 8 CTAs, 8 x 4096 fp64 bins distributed over their shared memory
+    CK(cudaFuncSetAttribute(red_dsmem, cudaFuncAttributeMaxDynamicSharedMemorySize, sb * 8));
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(nsm / 8 * 8 * 2);
+    cfg.blockDim = dim3(threads);
+    cfg.dynamicSmemBytes = sb * 8;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = 8;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    const float msd = t.best([&] { CK(cudaLaunchKernelEx(&cfg, red_dsmem, out, it, (uint32_t)sb)); });
+    CK(cudaGetLastError());
+    printf(" \"red_dsmem_f64_per_s\": %.4g,\n", (double)cfg.gridDim.x * threads * it / (msd * 1e-3));
   }
   {
     const int it = 4096;
