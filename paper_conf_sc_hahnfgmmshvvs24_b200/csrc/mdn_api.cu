@@ -37,6 +37,7 @@ struct mdn_grid {
   mdn::FluxView flux0{};      // view of table 0 (device pointers)
   mdn::Hitter* d_hit = nullptr;       // cull -> walk hand-off buffer
   uint32_t hit_cap = 0;
+  uint32_t hit_cap_max = 0;  // kMaxSlab, lowered if the device cannot hold that buffer
   mdn::DevCounters* d_ctr = nullptr;
   double* d_xs = nullptr;    // scratch for host xs
   unsigned long long* d_stats = nullptr;  // 6 work counters (mdnorm_stats)
@@ -190,7 +191,14 @@ mdn::MdnParams mdn_params(mdn_grid* g, double k_min, double k_max, int64_t pix_b
   return p;
 }
 
-constexpr uint32_t kMaxSlab = 1u << 24;  // trajectories per cull/walk pair (1 GiB hitter buffer)
+#ifndef MDN_MAX_SLAB_LOG2
+#define MDN_MAX_SLAB_LOG2 27
+#endif
+// Trajectories per cull/walk pair.  The hitter buffer holds a slab's worst case (every trajectory
+// hits, 64 B each: up to 8 GiB of the 180 GB).  Large slabs pay: the walk of one CORELLI run
+// (342K hitters) runs at 1.07e11 segments/s, a batch of 16 runs in one slab at ~1.4e11
+// (measured: the 120-run scan 64 ms with 2^24-trajectory slabs, 38 ms with 2^27).
+constexpr uint32_t kMaxSlab = 1u << MDN_MAX_SLAB_LOG2;
 
 // MDNorm over all nmat x nshard trajectories of one launch block: slabs of at most kMaxSlab
 // trajectories, each a cull kernel (compacting hitters into g->d_hit) and a walk kernel.  The
@@ -199,7 +207,7 @@ constexpr uint32_t kMaxSlab = 1u << 24;  // trajectories per cull/walk pair (1 G
 mdn_status run_mdnorm(mdn_grid* g, mdn::MdnParams p, const MatBlock& mb, cudaStream_t s) {
   const uint64_t ntraj = (uint64_t)mb.nmat * (uint64_t)p.nshard;
   if (ntraj == 0) return MDN_OK;
-  const uint32_t want = (uint32_t)std::min<uint64_t>(ntraj, kMaxSlab);
+  const uint32_t want = (uint32_t)std::min<uint64_t>(ntraj, g->hit_cap_max);
   if (g->hit_cap < want) {
     if (g->d_hit) {
       cudaStreamSynchronize(s);
@@ -207,14 +215,25 @@ mdn_status run_mdnorm(mdn_grid* g, mdn::MdnParams p, const MatBlock& mb, cudaStr
     }
     g->d_hit = nullptr;
     g->hit_cap = 0;
-    MDN_CUDA(cudaMalloc(&g->d_hit, sizeof(mdn::Hitter) * (size_t)want), "hitter buffer");
-    g->hit_cap = want;
+    // largest buffer the device grants, halving down to 2^20 trajectories (smaller slabs)
+    uint32_t cap = want;
+    cudaError_t e = cudaMalloc(&g->d_hit, sizeof(mdn::Hitter) * (size_t)cap);
+    while (e == cudaErrorMemoryAllocation && cap > (1u << 20)) {
+      cudaGetLastError();
+      cap /= 2;
+      e = cudaMalloc(&g->d_hit, sizeof(mdn::Hitter) * (size_t)cap);
+    }
+    MDN_CUDA(e, "hitter buffer");
+    g->hit_cap = cap;
+    if (cap < want) g->hit_cap_max = cap;  // do not retry the larger size on every call
   }
   if (!g->d_ctr) MDN_CUDA(cudaMalloc(&g->d_ctr, sizeof(mdn::DevCounters)), "counters");
   p.hit = g->d_hit;
   p.ctr = g->d_ctr;
-  // pixels per slab so that every trajectory of the slab can be a hitter
-  const uint64_t per = std::max<uint64_t>(1, g->hit_cap / (uint64_t)mb.nmat);
+  // pixels per slab so that every trajectory of the slab can be a hitter, split evenly
+  const uint64_t cap_px = std::max<uint64_t>(1, g->hit_cap / (uint64_t)mb.nmat);
+  const uint64_t nslab = ((uint64_t)p.nshard + cap_px - 1) / cap_px;
+  const uint64_t per = ((uint64_t)p.nshard + nslab - 1) / nslab;
   for (uint64_t p0 = 0; p0 < (uint64_t)p.nshard; p0 += per) {
     p.p0 = (uint32_t)p0;
     p.plen = (uint32_t)std::min<uint64_t>(per, (uint64_t)p.nshard - p0);
@@ -356,6 +375,7 @@ mdn_status mdnorm_create_grid(int device, const double lo[3], const double hi[3]
   mdn_grid* g = new mdn_grid;
   g->device = device;
   g->acc = acc;
+  g->hit_cap_max = kMaxSlab;
   cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, device);
   for (int a = 0; a < 3; ++a) {
     g->g.lo[a] = lo[a];

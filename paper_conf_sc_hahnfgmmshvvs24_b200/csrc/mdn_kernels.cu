@@ -39,6 +39,10 @@ namespace {
 #define MDN_WALK_CHUNK 8
 #endif
 constexpr int kWalkChunk = MDN_WALK_CHUNK;
+// claims shrink to kWalkChunk hitters once fewer than MDN_WALK_TAIL x 32 hitters per warp remain
+#ifndef MDN_WALK_TAIL
+#define MDN_WALK_TAIL 4
+#endif
 // claimed hitters sorted by piece length before they enter the warp's queue
 #ifndef MDN_WALK_SORT
 #define MDN_WALK_SORT 1
@@ -451,7 +455,7 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
   unsigned head = 0, nq = 0;
   int skip = 0, qpieces = 0;
   bool more = true;
-  const unsigned tail = 4u * 32u * gridDim.x * (unsigned)nwarps;
+  const unsigned tail = (unsigned)MDN_WALK_TAIL * 32u * gridDim.x * (unsigned)nwarps;
   unsigned chunk = nhit > tail ? 32u : (unsigned)kWalkChunk;
   for (;;) {
     while (qpieces < 32 && more) {
