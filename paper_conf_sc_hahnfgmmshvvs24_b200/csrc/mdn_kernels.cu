@@ -39,6 +39,13 @@ namespace {
 #define MDN_WALK_CHUNK 8
 #endif
 constexpr int kWalkChunk = MDN_WALK_CHUNK;
+// the last MDN_WALK_SPLIT_TAIL hitters per warp are cut into MDN_WALK_SPLIT x more pieces
+#ifndef MDN_WALK_SPLIT
+#define MDN_WALK_SPLIT 2
+#endif
+#ifndef MDN_WALK_SPLIT_TAIL
+#define MDN_WALK_SPLIT_TAIL 4  // measured: 4 > 8 > 16 > 32 (-1% CORELLI walk at 4), split 4 slower
+#endif
 // claims shrink to kWalkChunk hitters once fewer than MDN_WALK_TAIL x 32 hitters per warp remain
 #ifndef MDN_WALK_TAIL
 #define MDN_WALK_TAIL 4
@@ -457,6 +464,8 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
   bool more = true;
   const unsigned tail = (unsigned)MDN_WALK_TAIL * 32u * gridDim.x * (unsigned)nwarps;
   unsigned chunk = nhit > tail ? 32u : (unsigned)kWalkChunk;
+  const unsigned split_tail = (unsigned)MDN_WALK_SPLIT_TAIL * gridDim.x * (unsigned)nwarps;
+  (void)split_tail;
   for (;;) {
     while (qpieces < 32 && more) {
       unsigned b = 0;
@@ -480,6 +489,11 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
         const int4 t = *reinterpret_cast<const int4*>(&p.hit[b + lane].A);  // (A, jA, stepG, P)
         A = t.x;
         P = t.w;
+#if MDN_PIECE_BALANCED && MDN_WALK_SPLIT > 1
+        // the last hitters of the launch are cut into MDN_WALK_SPLIT times more (shorter) pieces
+        // at crossings of the same axis, so that the final rounds -- and the kernel -- end sooner
+        if (nhit - b <= split_tail) P = max(P, min(abs(t.z), P * MDN_WALK_SPLIT));
+#endif
       }
       unsigned key = (unsigned)lane < nnew ? ((((unsigned)A >> 22) + 1u) << 5) | (unsigned)lane : 0u;
 #pragma unroll
@@ -523,13 +537,14 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
     __syncwarp();
     const int nr = min(qpieces, 32);
     unsigned myh = 0;
-    int mypi = 0;
+    int mypi = 0, myP = 1;
     if (lane < nr) {
       int l = 0;  // owner: first queued hitter l with pre[l] > lane
 #pragma unroll
       for (int s = 16; s > 0; s >>= 1)
         if (pre[l + s - 1] <= lane) l += s;
       myh = ring[(head + l) & (kWalkRing - 1)];
+      myP = ringP[(head + l) & (kWalkRing - 1)];  // the piece count this hitter was queued with
       mypi = lane - (l ? pre[l - 1] : 0) + (l == 0 ? skip : 0);
     }
     // advance the queue past the nr pieces handed out
@@ -545,16 +560,16 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
       const double v0 = h.v0, v1 = h.v1, v2 = h.v2;
       const int A = h.A & 3;
       double lo_k = h.kin, hi_k = h.kout;
-      if (h.P > 1) {
+      if (myP > 1) {
         const double vA = A == 0 ? v0 : (A == 1 ? v1 : v2);
         const double rA = ddiv(1.0, vA);
 #if MDN_PIECE_BALANCED
         const int cA = abs(h.stepG), st = h.stepG < 0 ? -1 : 1;
-        if (mypi > 0) lo_k = plane_k(p.g, A, h.jA + st * ((mypi * cA) / h.P), rA);
-        if (mypi < h.P - 1) hi_k = plane_k(p.g, A, h.jA + st * (((mypi + 1) * cA) / h.P), rA);
+        if (mypi > 0) lo_k = plane_k(p.g, A, h.jA + st * ((mypi * cA) / myP), rA);
+        if (mypi < myP - 1) hi_k = plane_k(p.g, A, h.jA + st * (((mypi + 1) * cA) / myP), rA);
 #else
         if (mypi > 0) lo_k = plane_k(p.g, A, h.jA + mypi * h.stepG, rA);
-        if (mypi < h.P - 1) hi_k = plane_k(p.g, A, h.jA + (mypi + 1) * h.stepG, rA);
+        if (mypi < myP - 1) hi_k = plane_k(p.g, A, h.jA + (mypi + 1) * h.stepG, rA);
 #endif
       }
       int nc;
