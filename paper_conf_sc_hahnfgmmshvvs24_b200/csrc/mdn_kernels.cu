@@ -20,6 +20,10 @@
 
 namespace mdn {
 
+#if MDN_WALK_TRACE
+__device__ unsigned long long g_walk_trace[4 * 148 * 32];  // timing experiment (per walk warp)
+#endif
+
 namespace {
 
 // One persistent walk CTA per SM (the shared-memory flux table takes up to 196 KB): 1024
@@ -45,6 +49,15 @@ constexpr int kWalkChunk = MDN_WALK_CHUNK;
 #endif
 #ifndef MDN_WALK_SPLIT_TAIL
 #define MDN_WALK_SPLIT_TAIL 4  // measured: 4 > 8 > 16 > 32 (-1% CORELLI walk at 4), split 4 slower
+#endif
+#ifndef MDN_WALK_TRACE
+#define MDN_WALK_TRACE 0  // timing experiment: per-warp start / first round / end timestamps
+#endif
+#ifndef MDN_WALK_STATIC_PCT
+#define MDN_WALK_STATIC_PCT 60  // % of a launch's hitters in static per-CTA blocks
+#endif
+#ifndef MDN_WALK_STATIC_CHUNK
+#define MDN_WALK_STATIC_CHUNK 32  // hitters per claim from the CTA's block
 #endif
 // claims shrink to kWalkChunk hitters once fewer than MDN_WALK_TAIL x 32 hitters per warp remain
 #ifndef MDN_WALK_TAIL
@@ -437,7 +450,13 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
       sTab[i] = (uint16_t)((e & (kFluxDense32 - 1)) | ((e & kFluxDense32) ? kFluxDense16 : 0u));
     }
   }
+  __shared__ unsigned sCur;  // claims taken from this CTA's static block of hitters
+  if (threadIdx.x == 0) sCur = 0;
   __syncthreads();
+#if MDN_WALK_TRACE
+  unsigned long long tr_t0 = 0, tr_first = 0, tr_rounds = 0;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tr_t0));
+#endif
   FluxView fx = p.flux;
   if (kSmemFlux) {
     if (!MDN_FLUX_NOKN) fx.kn = sKn;  // else the rare general path bisects the global knots
@@ -464,21 +483,44 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
   bool more = true;
   const unsigned tail = (unsigned)MDN_WALK_TAIL * 32u * gridDim.x * (unsigned)nwarps;
   unsigned chunk = nhit > tail ? 32u : (unsigned)kWalkChunk;
+  // static per-CTA blocks of hitters cover MDN_WALK_STATIC_PCT % of them; [rest, nhit) is dynamic
+  // (only for launches small enough to claim in small chunks from the start: with 32-hitter
+  // claims the global counter is not contended, and static blocks unbalance 3-D walks)
+  const unsigned blk_n =
+      nhit > tail ? 0u : (unsigned)(((unsigned long long)nhit * MDN_WALK_STATIC_PCT / 100) / gridDim.x);
+  const unsigned blk = blockIdx.x * blk_n, rest = blk_n * gridDim.x;
+  constexpr int kStaticChunk = MDN_WALK_STATIC_CHUNK;
+  bool sdone = false;  // lane 0: this CTA's block is used up
   const unsigned split_tail = (unsigned)MDN_WALK_SPLIT_TAIL * gridDim.x * (unsigned)nwarps;
   (void)split_tail;
   for (;;) {
     while (qpieces < 32 && more) {
-      unsigned b = 0;
-      if (lane == 0) b = atomicAdd(&p.ctr->claimed, chunk);
+      // Claims come first from this CTA's static block of hitters (a shared-memory atomic), then
+      // from the launch's remaining hitters (one global atomic): the block keeps the 4736 warps
+      // from queueing on one global counter (at the start every warp claims at once, measured
+      // 10 us before the last warp's first round), the global remainder balances the CTAs.
+      unsigned b = 0, n = 0;
+      if (lane == 0) {
+        const unsigned o = sdone ? blk_n : atomicAdd(&sCur, (unsigned)kStaticChunk);
+        if (o < blk_n) {
+          b = blk + o;
+          n = min((unsigned)kStaticChunk, blk_n - o);
+        } else {
+          sdone = true;
+          b = rest + atomicAdd(&p.ctr->claimed, chunk);
+          n = chunk;
+        }
+      }
       b = __shfl_sync(kFull, b, 0);
+      n = __shfl_sync(kFull, n, 0);
       if (b >= nhit) {
         more = false;
         break;
       }
-      const unsigned nnew = min(chunk, nhit - b);
+      const unsigned nnew = min(n, nhit - b);
       // large claims (hitter locality, fewer atomics) until the last few claims per warp, then
       // small ones so that the warps finish together
-      chunk = nhit - b > tail ? 32u : (unsigned)kWalkChunk;
+      if (b >= rest) chunk = nhit - b > tail ? 32u : (unsigned)kWalkChunk;
       int P = 0;
 #if MDN_WALK_SORT
       // Claimed hitters enter the queue longest pieces first (warp bitonic sort on the piece
@@ -525,6 +567,9 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
       __syncwarp();
     }
     if (qpieces == 0) break;
+#if MDN_WALK_TRACE
+    if (tr_rounds++ == 0) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tr_first));
+#endif
     // pieces of the first (up to) 32 queued hitters: inclusive scan of their remaining counts
     const bool inq = (unsigned)lane < nq;
     int incl = inq ? ringP[(head + lane) & (kWalkRing - 1)] - (lane == 0 ? skip : 0) : 0;
@@ -590,6 +635,19 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
     __syncthreads();
     priv_flush(sHist, p.norm, p.g.nbins);
   }
+#if MDN_WALK_TRACE
+  if (lane == 0) {
+    unsigned long long t1;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t1));
+    unsigned long long* o = g_walk_trace + 4 * ((size_t)blockIdx.x * nwarps + warp);
+    o[0] = tr_t0;
+    o[1] = tr_first;
+    o[2] = t1;
+    unsigned smid;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+    o[3] = tr_rounds | ((unsigned long long)smid << 32);
+  }
+#endif
   if (kStats) flush_counter(p.stats + 3, c_seg);
 }
 
@@ -1167,4 +1225,11 @@ cudaError_t launch_debug_compose(const MatBlock& mdn, const MatBlock& bin, doubl
   return cudaGetLastError();
 }
 
+#if MDN_WALK_TRACE
+}  // namespace mdn
+extern "C" int mdn_debug_walk_trace(unsigned long long* out, int n) {
+  return (int)cudaMemcpyFromSymbol(out, mdn::g_walk_trace, sizeof(unsigned long long) * (size_t)n);
+}
+namespace mdn {
+#endif
 }  // namespace mdn
