@@ -13,6 +13,7 @@
 //   X2                xs_kernel
 // The parity entry points (debug_*) run the very same device functions (mdn_device.cuh).
 #include <algorithm>
+#include <cstdlib>
 #include <type_traits>
 
 #include "mdn_kernels.cuh"
@@ -515,6 +516,10 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
       n = __shfl_sync(kFull, n, 0);
       if (b >= nhit) {
         more = false;
+        // this warp claims nothing more: once every warp of every CTA is here (the start of the
+        // end spread) a BinMD launched with programmatic stream serialisation may take the SMs
+        // that walk CTAs leave
+        asm volatile("griddepcontrol.launch_dependents;");
         break;
       }
       const unsigned nnew = min(n, nhit - b);
@@ -912,6 +917,10 @@ binmd_kernel(const __grid_constant__ BinParams p, const __grid_constant__ MatBlo
     flush_counter(p.stats + 4, c_pairs);
     flush_counter(p.stats + 5, c_in);
   }
+  // Programmatic dependent launch (launch_binmd_t): this grid may start while the walk before it
+  // is still running (BinMD reads nothing the walk writes), but it does not complete before the
+  // walk has, so a kernel after BinMD still sees the norm histogram.  No-op without the attribute.
+  if (threadIdx.x == 0) asm volatile("griddepcontrol.wait;" ::: "memory");
 }
 
 // ---------------------------------------------------------------- X2
@@ -1090,8 +1099,22 @@ cudaError_t launch_binmd_t(const BinParams& p, const MatBlock& mb, int num_sms, 
   int per_sm = 0;
   err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, threads, smem);
   if (err != cudaSuccess) return err;
-  k<<<grid_for(p.nevents, num_sms, std::max(per_sm, 1), threads), threads, smem, s>>>(p, mb);
-  return cudaGetLastError();
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)grid_for(p.nevents, num_sms, std::max(per_sm, 1), threads));
+  cfg.blockDim = dim3(threads);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  // MDN_PDL=1 lets BinMD start during the preceding walk's end spread (programmatic dependent
+  // launch; see the end of binmd_kernel).  Off by default: measured on CORELLI 0.536 ms/step
+  // against 0.492 without -- BinMD's grid-stride CTAs get equal shares but start staggered over
+  // the walk's tail, so BinMD ends later than it gains.
+  static const bool pdl = [] { const char* e = std::getenv("MDN_PDL"); return e && std::atoi(e) != 0; }();
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = pdl ? 1 : 0;
+  return cudaLaunchKernelEx(&cfg, k, p, mb);
 }
 
 template <int kPriv>
