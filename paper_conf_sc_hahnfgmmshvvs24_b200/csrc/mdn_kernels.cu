@@ -251,6 +251,9 @@ mdnorm_cull_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ 
   double* sM = smem;
   double* sC = sM + 9 * mb.nmat;
   CullMat* sF = reinterpret_cast<CullMat*>(sC + mb.nmat);
+  // the walk (launched with programmatic stream serialisation, MDN_PDL_WALK) may start its
+  // prologue on SMs this one-wave grid leaves; it waits for this grid before reading hitters
+  asm volatile("griddepcontrol.launch_dependents;");
   stage_mdnorm_mats(mb, sM, sC);
   __syncthreads();
   // test order: fewest bins first (stable)
@@ -469,6 +472,10 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
   typename std::conditional<kPriv != 0, SmemEmit<PT>, AtomicEmit>::type emit;
   if constexpr (kPriv != 0) emit.h = sHist;
   else emit.h = p.norm;
+  // everything above (flux staging, private histogram zeroing) overlaps the cull's tail under
+  // programmatic dependent launch; the hitter list and count are read only after the cull
+  // grid has completed.  No-op without the attribute.
+  asm volatile("griddepcontrol.wait;" ::: "memory");
   const unsigned nhit = *(volatile unsigned*)&p.ctr->nhit;
   unsigned long long c_seg = 0;
   // Per-warp queue of hitters (ring of kWalkRing indices; the head hitter may be partly
@@ -1053,8 +1060,21 @@ cudaError_t launch_walk(const MdnParams& p, int num_sms, cudaStream_t s) {
   int per_sm = 0;
   err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, threads, smem);
   if (err != cudaSuccess) return err;
-  k<<<num_sms * std::max(per_sm, 1), threads, smem, s>>>(p);
-  return cudaGetLastError();
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)(num_sms * std::max(per_sm, 1)));
+  cfg.blockDim = dim3(threads);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  // programmatic dependent launch after the cull (see griddepcontrol.wait in mdnorm_walk_kernel):
+  // the walk's prologue and launch overlap the cull's tail.  Measured on CORELLI: MDNorm 0.362 ms
+  // vs 0.372, step 0.481 vs 0.490.  MDN_PDL_WALK=0 turns it off.
+  static const bool pdl = [] { const char* e = std::getenv("MDN_PDL_WALK"); return !e || std::atoi(e) != 0; }();
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = pdl ? 1 : 0;
+  return cudaLaunchKernelEx(&cfg, k, p);
 }
 
 template <int kFlux, int kPriv>
