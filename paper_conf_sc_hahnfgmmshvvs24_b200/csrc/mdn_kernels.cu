@@ -751,6 +751,9 @@ binmd_kernel(const __grid_constant__ BinParams p, const __grid_constant__ MatBlo
     priv_zero(hb, p.g.nbins);
     if (p.col_e >= 0) priv_zero(he, p.g.nbins);
   }
+  // the divide after BinMD (launch_cross_section, programmatic dependent launch) may launch now;
+  // it waits for this grid to complete before reading either histogram
+  asm volatile("griddepcontrol.launch_dependents;");
   stage_binmd_mats(mb, sN);
   __syncthreads();
   for (int i = threadIdx.x; i < 3 * mb.nmat; i += blockDim.x) {
@@ -934,6 +937,9 @@ binmd_kernel(const __grid_constant__ BinParams p, const __grid_constant__ MatBlo
 __global__ void __launch_bounds__(kThreads)
 xs_kernel(const double* __restrict__ norm, const double* __restrict__ binmd, double* __restrict__ xs,
           int64_t n) {
+  // launched with programmatic stream serialisation: the histograms are read only after the
+  // preceding grid has completed (no-op without the attribute)
+  asm volatile("griddepcontrol.wait;" ::: "memory");
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
     const double d = norm[i];
@@ -1236,8 +1242,18 @@ int last_binmd_path() { return g_last_binmd_path; }
 
 cudaError_t launch_cross_section(const double* norm, const double* binmd, double* xs, int64_t nbins,
                                  int num_sms, cudaStream_t s) {
-  xs_kernel<<<grid_for(nbins, num_sms, 8), kThreads, 0, s>>>(norm, binmd, xs, nbins);
-  return cudaGetLastError();
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)grid_for(nbins, num_sms, 8));
+  cfg.blockDim = dim3(kThreads);
+  cfg.stream = s;
+  // programmatic dependent launch after BinMD (MDN_PDL_XS=0 turns it off)
+  static const bool pdl = [] { const char* e = std::getenv("MDN_PDL_XS"); return !e || std::atoi(e) != 0; }();
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = pdl ? 1 : 0;
+  return cudaLaunchKernelEx(&cfg, xs_kernel, norm, binmd, xs, nbins);
 }
 
 cudaError_t launch_cross_section_err(const double* norm, const double* binmd, const double* err2, double* xs,
