@@ -78,7 +78,8 @@ mdn_status mdnorm_create_grid(int device, const double lo[3], const double hi[3]
 mdn_status mdnorm_destroy(mdn_grid *g);
 
 /* Detector table ("CORELLI 372K and TOPAZ 1.6M"; VanadiumFile P:428).
- * dir: double[npix][3] unit vectors sample->pixel, lab frame, beam = +z (host or device);
+ * dir: double[npix][3] unit vectors sample->pixel, lab frame, beam = +z (host or device; any
+ * finite vectors are accepted and used as given, q_p = z - d_p);
  * solid: double[npix] solid angle x vanadium factor, >= 0, 0 == masked pixel. */
 mdn_status mdnorm_set_instrument(mdn_grid *g, int64_t npix, const double *dir, const double *solid);
 
@@ -215,11 +216,24 @@ mdn_status mdnorm_debug_trajectories(mdn_grid *g, int32_t nmat, const double *M,
                                      int32_t *n_seg, int64_t *seg_bins, double *seg_vals,
                                      int64_t max_segs);
 
-/* Bin index (-1 = outside) of every (matrix, event) pair through the production BinMD index
- * code: bins[m * nevents + e] (HOST int64 array).  Synchronous. */
+/* Bin index (-1 = outside) of every (matrix, event) pair through the production BinMD decision
+ * (the same device functions as binmd_accumulate: op-class test, fp32 per-axis bins inside the
+ * proven error band, the exact fp64 formula for pairs within the band of a bin edge):
+ * bins[m * nevents + e] (HOST int64 array).  Synchronous. */
 mdn_status binmd_debug_bins(mdn_grid *g, int32_t nmat, const double *N, int64_t nevents,
                             const float *events, int64_t stride_floats, int32_t col_w,
                             int32_t col_q, int64_t *bins);
+
+/* Largest number of trajectories (matrix x pixel) per cull/walk slab of later MDNorm calls
+ * (max_traj in [1, 2^27]; 0 restores the default 2^27), so small inputs can exercise the
+ * multi-slab path.  No device work.  MDN_EINVAL: NULL grid or max_traj out of range. */
+mdn_status mdnorm_debug_set_max_slab(mdn_grid *g, int64_t max_traj);
+
+/* Launch facts of the last MDNorm call on g (HOST int64[4]): {slabs of its last launch block,
+ * hitters written by the cull of its last slab, the walk's large-launch threshold (hitters above
+ * which warps claim 32 hitters at a time with no static per-CTA blocks), the slab limit}.
+ * Synchronises the device. */
+mdn_status mdnorm_debug_last_launch(mdn_grid *g, int64_t out[4]);
 
 /* M_{r,s} / N_s exactly as the kernels compose them (device code; HOST outputs).  M: double
  * [nruns*nops][9] run-major; N: double[nops][9].  Synchronous (test entry point). */

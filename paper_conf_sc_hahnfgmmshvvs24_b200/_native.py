@@ -50,6 +50,8 @@ SIGNATURES = {
     "mdnorm_debug_trajectories": [P, i32, P, P, d, d, i64, P, P, P, P, P, i64],
     "binmd_debug_bins": [P, i32, P, i64, P, i64, i32, i32, P],
     "mdnorm_debug_compose": [P, P, i32, P, i32, P, P, P],
+    "mdnorm_debug_set_max_slab": [P, i64],
+    "mdnorm_debug_last_launch": [P, P],
 }
 _RESTYPES = {"mdn_last_error": C.c_char_p, "mdn_version": C.c_char_p}
 

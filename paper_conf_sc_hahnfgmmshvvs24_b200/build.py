@@ -37,18 +37,37 @@ def _stale() -> bool:
 
 def build(force: bool = False, verbose: bool = False, out: str | None = None,
           defines: tuple = ()) -> str:
-    """Compile libmdnorm.so.  out/defines build an experimental variant elsewhere (tools/)."""
+    """Compile libmdnorm.so: every .cu to an object in parallel (relocatable device code is not
+    needed: each translation unit owns its kernels), then one shared-library link.  out/defines
+    build an experimental variant elsewhere (tools/)."""
     target = out or LIB
     if out is None and not force and not _stale():
         return LIB
     nvcc = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
-    tmp = target + f".tmp{os.getpid()}"
-    cmd = [nvcc, *NVCC_FLAGS, *[f"-D{d}" for d in defines], "-I", INCLUDE, "-o", tmp, *sources()]
-    if verbose:
-        cmd.insert(1, "-Xptxas=-v")
-        print(" ".join(cmd), file=sys.stderr)
-    subprocess.check_call(cmd)
-    os.replace(tmp, target)
+    tag = f".tmp{os.getpid()}_{os.path.basename(target)}"
+    objs, procs = [], []
+    for src in sources():
+        obj = os.path.join(os.path.dirname(target), os.path.basename(src) + tag + ".o")
+        cmd = [nvcc, *NVCC_FLAGS, *[f"-D{d}" for d in defines], "-I", INCLUDE, "-c", "-o", obj, src]
+        cmd.remove("-shared")
+        if verbose:
+            cmd.insert(1, "-Xptxas=-v")
+            print(" ".join(cmd), file=sys.stderr)
+        objs.append(obj)
+        procs.append(subprocess.Popen(cmd))
+    try:
+        bad = [p.args for p in procs if p.wait() != 0]
+        if bad:
+            raise subprocess.CalledProcessError(1, bad[0])
+        tmp = target + tag
+        link = [nvcc, "-gencode", "arch=compute_100a,code=sm_100a", "-shared", "-cudart", "static",
+                "-Xcompiler", "-fPIC", "-o", tmp, *objs]
+        subprocess.check_call(link)
+        os.replace(tmp, target)
+    finally:
+        for o in objs:
+            if os.path.exists(o):
+                os.remove(o)
     return target
 
 

@@ -38,6 +38,9 @@ struct mdn_grid {
   mdn::Hitter* d_hit = nullptr;       // cull -> walk hand-off buffer
   uint32_t hit_cap = 0;
   uint32_t hit_cap_max = 0;  // kMaxSlab, lowered if the device cannot hold that buffer
+  uint32_t slab_limit = 0;   // trajectories per cull/walk slab (kMaxSlab; lowered by a test entry)
+  uint32_t last_nslab = 0;   // slabs of the last MDNorm launch block (tracing)
+  double qmax = 2.0;         // max(2, largest |q_p,i| of the instrument)
   mdn::DevCounters* d_ctr = nullptr;
   double* d_xs = nullptr;    // scratch for host xs
   unsigned long long* d_stats = nullptr;  // 6 work counters (mdnorm_stats)
@@ -184,6 +187,7 @@ mdn::MdnParams mdn_params(mdn_grid* g, double k_min, double k_max, int64_t pix_b
   p.priv = g->priv;
   p.kmin = k_min;
   p.kmax = k_max;
+  p.qmax = g->qmax;
   p.norm = g->d_hist;
   p.stats = g->stats_on ? g->d_stats : nullptr;
   p.hit = g->d_hit;
@@ -207,7 +211,7 @@ constexpr uint32_t kMaxSlab = 1u << MDN_MAX_SLAB_LOG2;
 mdn_status run_mdnorm(mdn_grid* g, mdn::MdnParams p, const MatBlock& mb, cudaStream_t s) {
   const uint64_t ntraj = (uint64_t)mb.nmat * (uint64_t)p.nshard;
   if (ntraj == 0) return MDN_OK;
-  const uint32_t want = (uint32_t)std::min<uint64_t>(ntraj, g->hit_cap_max);
+  const uint32_t want = (uint32_t)std::min<uint64_t>(ntraj, std::min(g->hit_cap_max, g->slab_limit));
   if (g->hit_cap < want) {
     if (g->d_hit) {
       cudaStreamSynchronize(s);
@@ -231,8 +235,9 @@ mdn_status run_mdnorm(mdn_grid* g, mdn::MdnParams p, const MatBlock& mb, cudaStr
   p.hit = g->d_hit;
   p.ctr = g->d_ctr;
   // pixels per slab so that every trajectory of the slab can be a hitter, split evenly
-  const uint64_t cap_px = std::max<uint64_t>(1, g->hit_cap / (uint64_t)mb.nmat);
+  const uint64_t cap_px = std::max<uint64_t>(1, std::min(g->hit_cap, g->slab_limit) / (uint64_t)mb.nmat);
   const uint64_t nslab = ((uint64_t)p.nshard + cap_px - 1) / cap_px;
+  g->last_nslab = (uint32_t)nslab;
   const uint64_t per = ((uint64_t)p.nshard + nslab - 1) / nslab;
   for (uint64_t p0 = 0; p0 < (uint64_t)p.nshard; p0 += per) {
     p.p0 = (uint32_t)p0;
@@ -273,7 +278,11 @@ mdn::BinParams bin_params(mdn_grid* g, const float* ev, int64_t n, const EvLayou
   // fp32 fast-path axis order: fewest bins first (stable), so a thin slab axis rejects early
   int ord[3] = {0, 1, 2};
   std::stable_sort(ord, ord + 3, [&](int a, int b) { return g->g.n[a] < g->g.n[b]; });
-  for (int a = 0; a < 3; ++a) p.ord[a] = ord[a];
+  const int32_t stride[3] = {1, g->g.n[0], g->g.n[0] * g->g.n[1]};
+  for (int a = 0; a < 3; ++a) {
+    p.ord[a] = ord[a];
+    p.st[a] = stride[ord[a]];
+  }
   p.acc_f32 = g->acc == MDN_ACC_F32;
   p.priv = g->priv;
   p.binmd = g->d_hist + g->g.nbins;
@@ -376,6 +385,7 @@ mdn_status mdnorm_create_grid(int device, const double lo[3], const double hi[3]
   g->device = device;
   g->acc = acc;
   g->hit_cap_max = kMaxSlab;
+  g->slab_limit = kMaxSlab;
   cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, device);
   for (int a = 0; a < 3; ++a) {
     g->g.lo[a] = lo[a];
@@ -433,6 +443,11 @@ mdn_status mdnorm_set_instrument(mdn_grid* g, int64_t npix, const double* dir, c
   MDN_CUDA(to_host(dir, 3 * npix, hd), "read dir");
   MDN_CUDA(to_host(solid, npix, hs), "read solid");
   if (!finite_all(hd.data(), 3 * npix)) return fail(MDN_EINVAL, "dir has non-finite values");
+  // the cull's fp32 pre-test band scales with the largest |q_i| = |(-d_x, -d_y, 1 - d_z)_i| (2 for
+  // unit directions): any direction table is accepted and decided exactly as the definition does
+  double qmax = 2.0;
+  for (int64_t i = 0; i < npix; ++i)
+    qmax = std::max(qmax, std::max(std::fabs(hd[3 * i]), std::max(std::fabs(hd[3 * i + 1]), std::fabs(1.0 - hd[3 * i + 2]))));
   for (int64_t i = 0; i < npix; ++i)
     if (!(std::isfinite(hs[i]) && hs[i] >= 0.0)) return fail(MDN_EINVAL, "solid[%lld] = %g is not >= 0", (long long)i, hs[i]);
   double *d_dir = nullptr, *d_sol = nullptr;
@@ -466,6 +481,7 @@ mdn_status mdnorm_set_instrument(mdn_grid* g, int64_t npix, const double* dir, c
   }
   g->d_pix = d_pix;
   g->npix = npix;
+  g->qmax = qmax;
   return ok();
 }
 
@@ -984,6 +1000,29 @@ mdn_status binmd_debug_bins(mdn_grid* g, int32_t nmat, const double* N, int64_t 
   cudaFree(d_ev);
   cudaFree(d_bins);
   if (e != cudaSuccess) return cuda_fail(e, "debug bins");
+  return ok();
+}
+
+mdn_status mdnorm_debug_set_max_slab(mdn_grid* g, int64_t max_traj) {
+  if (!g) return fail(MDN_EINVAL, "grid is NULL");
+  if (max_traj < 0 || max_traj > (int64_t)kMaxSlab)
+    return fail(MDN_EINVAL, "max_traj %lld outside [0, %u]", (long long)max_traj, kMaxSlab);
+  g->slab_limit = max_traj == 0 ? kMaxSlab : (uint32_t)max_traj;
+  return ok();
+}
+
+mdn_status mdnorm_debug_last_launch(mdn_grid* g, int64_t out[4]) {
+  if (!g || !out) return fail(MDN_EINVAL, "NULL argument");
+  DeviceGuard dg(g->device);
+  mdn::DevCounters c{};
+  if (g->d_ctr) {
+    MDN_CUDA(cudaDeviceSynchronize(), "sync");
+    MDN_CUDA(cudaMemcpy(&c, g->d_ctr, sizeof c, cudaMemcpyDeviceToHost), "counters D2H");
+  }
+  out[0] = g->last_nslab;
+  out[1] = c.nhit;
+  out[2] = mdn::walk_big_claim_threshold(g->g.n[2] > 1, g->num_sms);
+  out[3] = g->slab_limit;
   return ok();
 }
 

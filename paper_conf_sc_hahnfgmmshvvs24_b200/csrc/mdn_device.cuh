@@ -12,10 +12,6 @@
 #include <cuda_runtime.h>
 #include <math_constants.h>
 
-#ifndef MDN_MERGE2D_SELECT
-#define MDN_MERGE2D_SELECT 0  // 2-D slices: select-based two-stream merge (default: branch)
-#endif
-
 namespace mdn {
 
 // ------------------------------------------------------------------------------ grid constants
@@ -54,7 +50,25 @@ __device__ __forceinline__ void matmul3(const double* A, const double* B, double
                           dmul(A[3 * i + 2], B[6 + j]));
 }
 
-// out = adj(C)/det * scale, out_ij = (cof_ji / det) * scale.  Returns false if singular.
+// RN(a / b) from y = RN(1 / b) by Markstein's correction: q = RN(a y) is within one ulp of a / b,
+// r = a - q b is exact (one FMA) and RN(q + r y) is the correctly rounded quotient -- the same
+// argument as the flux interpolation below (tests/test_flux_division.py pins it).  Valid when a,
+// b and a / b are normal and far from overflow; callers check the range and otherwise divide.  A
+// zero numerator gives the quotient's signed zero directly.
+__device__ __forceinline__ double div_rn_recip(double a, double b, double y) {
+  if (a == 0.0) return dmul(a, y);
+  const double q = dmul(a, y);
+  const double r = __fma_rn(-q, b, a);
+  return __fma_rn(r, y, q);
+}
+
+__device__ __forceinline__ bool recip_range(double x) {
+  const double ax = fabs(x);
+  return ax == 0.0 || (ax > 0x1p-400 && ax < 0x1p400);
+}
+
+// out = adj(C)/det * scale, out_ij = (cof_ji / det) * scale.  Returns false if singular.  The nine
+// quotients share one IEEE reciprocal of det (div_rn_recip; bit-identical to nine divisions).
 __device__ __forceinline__ bool inv3_scaled(const double* C, double scale, double* out) {
   double cof[9];
   cof[0] = dsub(dmul(C[4], C[8]), dmul(C[5], C[7]));
@@ -68,14 +82,20 @@ __device__ __forceinline__ bool inv3_scaled(const double* C, double scale, doubl
   cof[8] = dsub(dmul(C[0], C[4]), dmul(C[1], C[3]));
   double det = dadd(dadd(dmul(C[0], cof[0]), dmul(C[1], cof[1])), dmul(C[2], cof[2]));
   if (det == 0.0 || !isfinite(det)) return false;
+  const double y = ddiv(1.0, det);
+  bool fast = recip_range(det);
+#pragma unroll
+  for (int i = 0; i < 9; ++i) fast = fast && recip_range(cof[i]);
 #pragma unroll
   for (int i = 0; i < 3; ++i)
 #pragma unroll
-    for (int j = 0; j < 3; ++j) out[3 * i + j] = dmul(ddiv(cof[3 * j + i], det), scale);
+    for (int j = 0; j < 3; ++j)
+      out[3 * i + j] = dmul(fast ? div_rn_recip(cof[3 * j + i], det, y) : ddiv(cof[3 * j + i], det), scale);
   return true;
 }
 
-__device__ __forceinline__ double inv_two_pi() { return ddiv(1.0, dmul(2.0, CUDART_PI)); }
+// RN(1 / RN(2 pi)) (0x3fc45f306dc9c883), the constant the oracle's 1.0 / (2.0 * pi) evaluates to
+__device__ __forceinline__ double inv_two_pi() { return __hiloint2double(0x3fc45f30, 0x6dc9c883); }
 
 // M_{r,s} = (R UB S W)^-1 / (2 pi)   (reading #1-#2; rotations P:80, per-op 3x3 P:143/148)
 __device__ __forceinline__ bool compose_mdnorm(const double* R, const double* UB, const double* S,
@@ -121,16 +141,13 @@ __device__ __forceinline__ bool compose_binmd(const double* UB, const double* S,
 // than three knots (and c = 0, x outside the table, or c + 1 > U_{n-1}) are flagged and take the
 // general path: clamps and a bisection.  A fast cell lies below U_{n-1}, so its probes stop at
 // kappa_{n-1} at the latest: they read kappa_{i+1} from the next interval record (ka[n-1] holds
-// kappa_{n-1}), and the shared-memory copy needs no separate knot array (MDN_FLUX_NOKN; the
-// freed 32 KB pay for the 8 cells per knot: measured 1-2% faster walk than 4 cells + knots).
+// kappa_{n-1}), and the shared-memory copy needs no separate knot array (the freed 32 KB pay for
+// the 8 cells per knot: measured 1-2% faster walk than 4 cells + knots).
 // The general path bisects the global knot array (two +inf pads).
 //
 // Shared-memory layout (bank conflicts of random look-ups, measured: profiles/): the two records as separate
 // 16-byte-strided double2 arrays (all 8 sixteen-byte bank groups), instead of one 32-byte record
 // per interval (which uses only 4 of the 8 groups).
-#ifndef MDN_FLUX_NOKN
-#define MDN_FLUX_NOKN 1  // no shared-memory knot array: probes read the next interval record (frees 32 KB)
-#endif
 #ifndef MDN_FLUX_CELLS
 #define MDN_FLUX_CELLS 8  // cell-table cells per knot (at least); measured 8 > 6 > 4 with MDN_FLUX_NOKN
 #endif
@@ -176,30 +193,19 @@ __device__ __forceinline__ double flux_general(const FluxView& f, double x) {
 
 template <typename TabT = int>
 __device__ __forceinline__ double flux_at(const FluxView& f, double x) {
-#ifdef MDN_EXP_NOFLUX  // timing experiment only (wrong results): F(x) = x
-  return x;
-#endif
   constexpr unsigned flag = sizeof(TabT) == 2 ? kFluxDense16 : kFluxDense32;
   const int c = __double2int_rd(dmul(dsub(x, f.k_first), f.inv_cell));
   const unsigned e = (unsigned)c < (unsigned)f.ntab ? tab_entry<TabT>(f, c) : flag;
   if (e & flag) return flux_general(f, x);
   int i = (int)e;
-  // kappa_{i+1}: from the knot array, or (MDN_FLUX_NOKN) from the next interval record -- the
-  // fast path never looks past kappa_{n-1} (its cells end below U_{n-1})
-#if MDN_FLUX_NOKN
+  // kappa_{i+1} from the next interval record: the fast path never looks past kappa_{n-1} (its
+  // cells end below U_{n-1})
   double kn1 = f.ka[i + 1].x;
-#else
-  double kn1 = f.kn[i + 1];
-#endif
   double2 a = f.ka[i], b = f.kb[i];
   if (kn1 <= x) {  // a knot of cell c lies at or below x (at most three)
     do {
       ++i;
-#if MDN_FLUX_NOKN
       kn1 = f.ka[i + 1].x;
-#else
-      kn1 = f.kn[i + 1];
-#endif
     } while (kn1 <= x);
     a = f.ka[i];
     b = f.kb[i];

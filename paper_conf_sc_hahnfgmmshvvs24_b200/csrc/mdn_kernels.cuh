@@ -73,6 +73,7 @@ struct MdnParams {
   int32_t acc_f32;         // privatised partial sums in fp32 (MDN_ACC_F32) instead of fp64
   int32_t priv;            // shared-memory privatised histogram: -1 auto, 0 never, 1 whenever it fits
   double kmin, kmax;
+  double qmax;             // max(2, max_p max_i |q_p,i|): scales the cull's fp32 error band
   double* norm;            // fp64 histogram (nbins)
   unsigned long long* stats;  // nullptr, or [traj, hits, crossings, segments] (+= per launch)
   // cull -> walk hand-off (production path)
@@ -88,6 +89,7 @@ struct BinParams {
   int32_t col_w, col_q;
   int32_t col_e;           // error-squared column, or -1
   int32_t ord[3];          // axis test order of the fp32 fast path (fewest bins first)
+  int32_t st[3];           // linear-index stride of axis ord[k] (1, n0, n0 n1)
   int32_t acc_f32;         // privatised partial sums in fp32 (MDN_ACC_F32) instead of fp64
   int32_t priv;            // shared-memory privatised histogram: -1 auto, 0 never, 1 whenever it fits
   double* binmd;           // fp64 histogram (nbins)
@@ -100,6 +102,9 @@ cudaError_t launch_pixels_prepare(const double* dir, const double* solid, double
                                   cudaStream_t s);
 // MDNorm for shard pixels [p.p0, p.p0 + p.plen) x all matrices: cull (M1-M3) + piece walk (M3-M7).
 cudaError_t launch_mdnorm(const MdnParams& p, const MatBlock& mb, int num_sms, cudaStream_t s);
+// Hitters per walk launch above which warps claim 32 hitters at a time from the start (no static
+// per-CTA blocks): the walk's large-launch regime (tests assert they cover it).
+uint32_t walk_big_claim_threshold(bool d3, int num_sms);
 cudaError_t launch_binmd(const BinParams& p, const MatBlock& mb, int num_sms, cudaStream_t s);
 // Accumulation path chosen for the last launch_mdnorm / launch_binmd on this thread (tracing and
 // tests): 0 = global fp64 red.add, 1 = shared-memory fp64 partials, 2 = shared-memory fp32 partials.

@@ -55,21 +55,6 @@ struct WalkState {
     if (left == 0) return hi_k;
     --left;
     if (!k3D) {  // 2-D slice: two streams
-#if MDN_MERGE2D_SELECT
-      const bool p0 = c0.nk <= c1.nk;
-      const double k = p0 ? c0.nk : c1.nk;
-      const double jd = p0 ? c0.jd + c0.stepd : c1.jd + c1.stepd;
-      const int cnt = (p0 ? c0.cnt : c1.cnt) - 1;
-      const double nk = cnt > 0 ? dmul(dadd(p0 ? g.lo[0] : g.lo[1], dmul(jd, p0 ? g.w[0] : g.w[1])), p0 ? c0.r : c1.r)
-                                : CUDART_INF;
-      c0.jd = p0 ? jd : c0.jd;
-      c0.cnt = p0 ? cnt : c0.cnt;
-      c0.nk = p0 ? nk : c0.nk;
-      c1.jd = p0 ? c1.jd : jd;
-      c1.cnt = p0 ? c1.cnt : cnt;
-      c1.nk = p0 ? c1.nk : nk;
-      return k;
-#else
       if (c0.nk <= c1.nk) {
         const double k = c0.nk;
         c0.jd += c0.stepd;
@@ -82,7 +67,6 @@ struct WalkState {
       --c1.cnt;
       c1.nk = c1.cnt > 0 ? dmul(dadd(g.lo[1], dmul(c1.jd, g.w[1])), c1.r) : CUDART_INF;
       return k;
-#endif
     }
     // three streams, selects only: advance the chosen axis with one plane evaluation
     const bool s01 = c1.nk < c0.nk;

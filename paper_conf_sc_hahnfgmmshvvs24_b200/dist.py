@@ -7,7 +7,7 @@ function is used to add histograms").  Here:
   * a single run  -> pixels interleaved by rank (p = rank, rank + G, ...) so every GPU sees every
     detector region (balances the CORELLI slab, where only ~4% of trajectories hit the grid),
     and that run's events split into contiguous ranges;
-  * exchange      -> ONE collective over the packed fp64 [norm | binmd] buffer (sum); rank 0
+  * exchange      -> ONE collective over the packed fp64 [norm | binmd (| err2)] buffer (sum); rank 0
     (or every rank for all_reduce) then divides -- or, for grids too large to gather on one
     GPU (the 500^3 stress grid: 2 GB packed), ONE reduce_scatter that leaves every rank the summed
     norm and binmd of its own contiguous bin block, which it divides locally (mdn_divide).
@@ -57,50 +57,68 @@ def plan_shards(world: int, rank: int, nruns: int, npix: int, events_per_run) ->
     return p
 
 
-def reduce_packed(packed, group=None, dst: int | None = 0):
-    """Sum the packed [norm | binmd] histograms of all ranks with one collective.
+def _halves(packed, nbins: int | None, with_err: bool):
+    """The prefix of the packed [norm | binmd | err2] buffer one collective must cover: norm and
+    binmd (2 nbins doubles), plus err2 only when the error column was accumulated."""
+    n = packed.numel() // 3 if nbins is None else int(nbins)
+    if packed.numel() < 3 * n:
+        raise ValueError(f"packed buffer holds {packed.numel()} doubles, need 3 * nbins = {3 * n}")
+    return n, packed[: (3 if with_err else 2) * n]
 
-    dst=None -> all_reduce (every rank gets the sum); otherwise reduce to rank `dst`."""
+
+def reduce_packed(packed, group=None, dst: int | None = 0, nbins: int | None = None,
+                  with_err: bool = False):
+    """Sum the library's packed [norm | binmd | err2] histograms (3 * nbins doubles, as
+    `packed_histograms` returns them) of all ranks with ONE collective, in place.
+
+    Only [norm | binmd] travels unless with_err (binmd_accumulate_err was used): err2 is
+    otherwise all zero.  dst=None -> all_reduce (every rank gets the sum); otherwise reduce to
+    rank `dst`.  nbins defaults to numel // 3."""
     import torch.distributed as dist
+    n, view = _halves(packed, nbins, with_err)
     if not dist.is_available() or not dist.is_initialized() or dist.get_world_size(group) == 1:
         return packed
-    buf = packed
-    if packed.is_cuda and dist.get_backend(group) == "gloo":  # gloo (CPU tests): host staging
-        buf = packed.cpu()
+    buf = view
+    if view.is_cuda and dist.get_backend(group) == "gloo":  # gloo (CPU tests): host staging
+        buf = view.cpu()
     if dst is None:
         dist.all_reduce(buf, op=dist.ReduceOp.SUM, group=group)
     else:
         dist.reduce(buf, dst=dst, op=dist.ReduceOp.SUM, group=group)
-    if buf is not packed:
-        packed.copy_(buf)
+    if buf is not view:
+        view.copy_(buf)
     return packed
 
 
-def reduce_scatter_packed(packed, group=None):
-    """Sum the packed [norm | binmd] histograms of all ranks with ONE reduce_scatter; rank r gets
-    bins [b0, b1) (contiguous blocks of ceil(nbins / world)) of both halves.
+def reduce_scatter_packed(packed, group=None, nbins: int | None = None, with_err: bool = False):
+    """Sum the library's packed [norm | binmd | err2] histograms of all ranks with ONE
+    reduce_scatter; rank r gets bins [b0, b1) (contiguous blocks of ceil(nbins / world)) of norm
+    and binmd (and err2 when with_err).
 
-    Returns (norm_shard, binmd_shard, (b0, b1)) -- views of a new buffer; divide them with
-    mdn_divide.  The bin blocks are laid out rank-major ([rank][norm|binmd][block], zero padded)
-    before the collective so that each rank's output is [norm block | binmd block]."""
-    import torch
+    Returns (norm_shard, binmd_shard, (b0, b1)), or (norm_shard, binmd_shard, err2_shard, (b0, b1))
+    when with_err -- views of a new buffer; divide them with mdn_divide.  The bin blocks are laid
+    out rank-major ([rank][part][block], zero padded) before the collective so that each rank's
+    output is [norm block | binmd block (| err2 block)]."""
     import torch.distributed as dist
-    n = packed.numel() // 2
+    n, _ = _halves(packed, nbins, with_err)
+    parts = 3 if with_err else 2
     if not dist.is_available() or not dist.is_initialized() or dist.get_world_size(group) == 1:
-        return packed[:n], packed[n:2 * n], (0, n)
+        views = tuple(packed[i * n:(i + 1) * n] for i in range(parts))
+        return (*views, (0, n))
     world, rank = dist.get_world_size(group), dist.get_rank(group)
     chunk = -(-n // world)
-    tmp = packed.new_zeros(2, world * chunk)
-    tmp[0, :n] = packed[:n]
-    tmp[1, :n] = packed[n:2 * n]
-    src = tmp.view(2, world, chunk).transpose(0, 1).contiguous().view(-1)  # [rank][half][block]
-    out = packed.new_empty(2 * chunk)
+    tmp = packed.new_zeros(parts, world * chunk)
+    for i in range(parts):
+        tmp[i, :n] = packed[i * n:(i + 1) * n]
+    src = tmp.view(parts, world, chunk).transpose(0, 1).contiguous().view(-1)  # [rank][part][block]
+    out = packed.new_empty(parts * chunk)
     if dist.get_backend(group) == "gloo":  # gloo (CPU tests) has no reduce_scatter: all_reduce + slice
         buf = src.cpu() if src.is_cuda else src
         dist.all_reduce(buf, op=dist.ReduceOp.SUM, group=group)
-        out.copy_(buf.view(world, 2 * chunk)[rank])
+        out.copy_(buf.view(world, parts * chunk)[rank])
     else:
         dist.reduce_scatter_tensor(out, src, op=dist.ReduceOp.SUM, group=group)
     b0 = min(n, rank * chunk)
     b1 = min(n, b0 + chunk)
-    return out[: b1 - b0], out[chunk: chunk + b1 - b0], (b0, b1)
+    views = tuple(out[i * chunk: i * chunk + b1 - b0] for i in range(parts))
+    return (*views, (b0, b1))

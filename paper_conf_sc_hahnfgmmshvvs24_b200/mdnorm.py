@@ -363,3 +363,15 @@ def mdnorm_debug_compose(g: Grid, UB, R, ops):
                                       ops.ctypes.data, M.ctypes.data, N.ctypes.data),
           "mdnorm_debug_compose")
     return M.reshape(-1, 3, 3), N.reshape(-1, 3, 3)
+
+
+def mdnorm_debug_set_max_slab(g: Grid, max_traj: int) -> None:
+    """Trajectories per cull/walk slab of later MDNorm calls (0 = default 2^27)."""
+    check(load().mdnorm_debug_set_max_slab(g.handle, int(max_traj)), "mdnorm_debug_set_max_slab")
+
+
+def mdnorm_debug_last_launch(g: Grid) -> dict:
+    """{slabs, hitters (last slab), big_claim_threshold, slab_limit} of the last MDNorm call."""
+    out = np.zeros(4, np.int64)
+    check(load().mdnorm_debug_last_launch(g.handle, out.ctypes.data), "mdnorm_debug_last_launch")
+    return dict(zip(("slabs", "hitters", "big_claim_threshold", "slab_limit"), (int(x) for x in out)))

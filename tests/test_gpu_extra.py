@@ -177,13 +177,91 @@ def test_two_processes_one_gpu_reduce(mdn):
     assert np.array_equal(np.isnan(xs), np.isnan(oxs))
 
 
+def _rs_dist_worker(rank, world, port, q):
+    """reduce_scatter of the library's real 3-part buffer [norm | binmd | err2] (err2 written by
+    binmd_accumulate_err), then mdn_divide on each rank's own bin block."""
+    import torch
+    import torch.distributed as dist
+    sys.path.insert(0, ROOT)
+    import paper_conf_sc_hahnfgmmshvvs24_b200 as m
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    wl = synth.make_workload("corelli", events_per_run=300_000)
+    ev = synth.events_for_run(wl, 0)
+    ev8 = np.zeros((len(ev), 8), np.float32)
+    ev8[:, 0] = ev[:, 0]
+    ev8[:, 1] = 0.5 * ev[:, 0] + 0.25
+    ev8[:, 5:8] = ev[:, 1:4]
+    nb = [61, 47, 1]  # 2867 bins: not a multiple of the world size (padded blocks)
+    plan = m.plan_shards(world, rank, 1, wl.npix, len(ev))
+    g = m.mdnorm_create_grid(0, wl.lo, wl.hi, nb, wl.W)
+    m.mdnorm_set_privatization(g, m.MDN_PRIV_OFF)
+    m.mdnorm_set_instrument(g, wl.pix_dir, wl.solid)
+    m.mdnorm_set_flux(g, wl.flux_k, wl.flux_F)
+    m.mdnorm_accumulate(g, wl.UB, wl.R[0], wl.ops, wl.k_min, wl.k_max, 1.0,
+                        pix_begin=plan.pix_begin, pix_stride=plan.pix_stride * 7)
+    b, e = plan.event_ranges[0]
+    m.binmd_accumulate_err(g, wl.UB, wl.ops, torch.from_numpy(ev8[b:e]).cuda(), col_w=0, col_e=1, col_q=5)
+    packed = m.packed_histograms(g)
+    ns, bs, es, (b0, b1) = m.reduce_scatter_packed(packed, nbins=g.nbins_total, with_err=True)
+    xs = m.mdn_divide(ns.contiguous(), bs.contiguous())
+    torch.cuda.synchronize()
+    q.put((rank, b0, b1, ns.cpu().numpy(), bs.cpu().numpy(), es.cpu().numpy(), xs.cpu().numpy()))
+    dist.barrier()
+    g.close()
+    dist.destroy_process_group()
+
+
+def test_two_processes_reduce_scatter_real_buffer(mdn):
+    """The reduce_scatter path (grids too large to gather) on the library's own
+    packed [norm | binmd | err2] buffer: every rank's norm, binmd and err2 blocks equal the
+    oracle's, and its divided block equals the oracle's xs (NaN masks equal)."""
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_rs_dist_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    res = sorted(q.get(timeout=600) for _ in range(2))
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    wl = synth.make_workload("corelli", events_per_run=300_000)
+    ev = synth.events_for_run(wl, 0)
+    ev8 = np.zeros((len(ev), 8), np.float32)
+    ev8[:, 0] = ev[:, 0]
+    ev8[:, 1] = 0.5 * ev[:, 0] + 0.25
+    ev8[:, 5:8] = ev[:, 1:4]
+    og = oracle.Grid(wl.lo, wl.hi, [61, 47, 1])
+    M = oracle.mdnorm_matrices(wl.R, wl.UB, wl.ops, wl.W)
+    onorm = oracle.Accumulator(og.nbins)
+    for r in range(2):
+        oracle.mdnorm(og, wl.pix_dir, wl.solid, wl.flux_k, wl.flux_F, M, 1.0, wl.k_min, wl.k_max,
+                      pix_begin=r, pix_stride=14, acc=onorm)
+    N = oracle.binmd_matrices(wl.UB, wl.ops, wl.W)
+    obm = oracle.binmd(og, N, ev8, col_w=0, col_q=5)
+    oe2 = oracle.binmd_err(og, N, ev8, col_e=1, col_q=5)
+    onorm = onorm.value()
+    oxs = oracle.cross_section(obm, onorm)
+    assert res[0][1] == 0 and res[0][2] == res[1][1] and res[1][2] == og.nbins
+    for rank, b0, b1, ns, bs, es, xs in res:
+        _assert_rel(ns, onorm[b0:b1])
+        _assert_rel(bs, obm[b0:b1])
+        _assert_rel(es, oe2[b0:b1])
+        assert np.array_equal(np.isnan(xs), np.isnan(oxs[b0:b1]))
+        fin = ~np.isnan(xs)
+        assert np.all(np.abs(xs[fin] - oxs[b0:b1][fin]) <= 3e-12 * np.abs(oxs[b0:b1][fin]))
+
+
 def test_bench_multi_rank_code_path():
-    """bench.py under torchrun with 2 ranks (gloo, both on GPU 0): the N > 1 code path runs and
-    rank 0 prints one JSON line with n_gpus = 2 (a code-path check, not a performance number)."""
+    """`bench.py --gpus 2` without torchrun launches its own 2 ranks (MDN_BENCH_SHARED_GPU=1: both
+    on GPU 0 over gloo): the N > 1 code path runs and rank 0 prints one JSON line with n_gpus = 2
+    (a code-path check, not a performance number)."""
     env = dict(os.environ, MDN_BENCH_SHARED_GPU="1")
-    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
-           "--master-addr", "127.0.0.1", "--master-port", str(_free_port()), os.path.join(ROOT, "bench.py"),
-           "--gpus", "2", "--steps", "2", "--warmup", "1", "--no-cpu-baseline", "--dist-backend", "gloo"]
+    env.pop("WORLD_SIZE", None)
+    cmd = [sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2", "--steps", "2", "--warmup", "3",
+           "--no-cpu-baseline"]
     r = subprocess.run(cmd, env=env, capture_output=True, text=True, timeout=900, cwd=ROOT)
     assert r.returncode == 0, r.stderr[-3000:]
     lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
