@@ -1,8 +1,8 @@
 #!/usr/bin/env python
 """Benchmark of the MDNorm + BinMD cross-section hot path (BASELINE.json metric).
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
-  (N > 1: launched by torchrun, one process per GPU, NCCL)
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--config C]
+  (N > 1: one process per GPU over NCCL -- under torchrun, or launched by bench.py itself)
 
 Workload (BASELINE.json configs[1], the config the metric is quoted on):
 CORELLI-shaped single run -- 372,736 pixels x 24 symmetry ops (6/mmm) = 8,945,664
@@ -188,6 +188,7 @@ def run_reference(args, rank, world):
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
             "data": "synthetic (seeded, SURVEY.md §8(d) recipe)", "config": config_dict(wl, 1),
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle",
+                             "cpu": host_cpu_info(),
                              "sample": f"every {stride}th pixel (all 24 ops) and every {stride}th event "
                                        f"of the CORELLI-shaped run per step; the C oracle on {threads} host "
                                        f"threads ({host_cpu()}), private histograms per thread"},
@@ -264,7 +265,9 @@ def cpu_baseline(wl, ev, stride):
     traj = wl.npix * wl.nops / stride
     # single-thread figure on an 8x smaller sample of the same run
     s1_md, s1_bm, _, _ = oracle_timed(wl, ev, 8 * stride, 1)
+    cpu = host_cpu_info()
     return {"value": traj / secs, "unit": UNIT, "cores": threads, "kind": "oracle",
+            "cpu": cpu,
             "sample": f"every {stride}th pixel (all {wl.nops} ops) + every {stride}th event of run 0 "
                       f"({traj:.0f} trajectories, {len(ev) // stride} events; "
                       f"MDNorm {t_md:.2f} s + BinMD {t_bm:.2f} s) on {threads} host threads "
@@ -277,74 +280,164 @@ def cpu_baseline(wl, ev, stride):
 # ----------------------------------------------------------------------------- our arm
 
 
-def run_ours(args, rank, world, local_rank):
-    import torch
-    import torch.distributed as dist
-    import synth
-    import paper_conf_sc_hahnfgmmshvvs24_b200 as m
-    from paper_conf_sc_hahnfgmmshvvs24_b200 import build
+def host_cpu_info() -> dict:
+    """CPU model, sockets, physical cores and the threads this process may use (S§8(d))."""
+    info = {"model": host_cpu(), "threads_available": host_threads()}
+    phys, sockets = set(), set()
+    try:
+        cur = {}
+        for line in open("/proc/cpuinfo"):
+            if not line.strip():
+                if "physical id" in cur and "core id" in cur:
+                    phys.add((cur["physical id"], cur["core id"]))
+                    sockets.add(cur["physical id"])
+                cur = {}
+                continue
+            k, _, v = line.partition(":")
+            cur[k.strip()] = v.strip()
+    except OSError:
+        pass
+    info["sockets"] = len(sockets) or None
+    info["physical_cores"] = len(phys) or None
+    return info
 
-    build.build()
-    torch.cuda.set_device(local_rank)
-    dev = torch.device("cuda", local_rank)
-    wl = make_bench_workload(world)
-    run = rank if world > 1 else 0
-    ev = synth.events_for_run(wl, run)
-    g = m.mdnorm_create_grid(local_rank, wl.lo, wl.hi, wl.nbins, wl.W, m.MDN_ACC_F64)
-    m.mdnorm_set_instrument(g, wl.pix_dir, wl.solid)
-    m.mdnorm_set_flux(g, wl.flux_k, wl.flux_F)
-    ev_dev = torch.from_numpy(ev).to(dev)
-    packed = m.packed_histograms(g)
-    xs_dev = torch.empty(g.nbins_total, dtype=torch.float64, device=dev)
-    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
-    R, c = wl.R[run], float(wl.charge[run])
 
-    def step(ph):
-        # ph: five phase events, or None (the headline pass: an event recorded between two
-        # kernels costs a few microseconds of stream serialisation, ~4% of this step)
+class Case:
+    """One bench workload on this rank: its grid, its runs, its device events and the step."""
+
+    def __init__(self, m, torch, synth, name, world, rank, local_rank, dev, nops=None):
+        self.name, self.world, self.rank = name, world, rank
+        if name == "corelli":
+            # configs[1]; weak scaling: rank r processes run r of a rotation scan (omega = 17 + 3r)
+            wl = synth.make_workload("corelli")
+            if world > 1:
+                wl.R = np.stack([synth.rot_y(17.0 + 3.0 * r) for r in range(world)])
+                wl.charge = np.ones(world)
+            self.runs = [rank if world > 1 else 0]
+            self.scaling = "weak"
+            ev = synth.events_for_run(wl, self.runs[0])
+            self.ev_dev = torch.from_numpy(ev).to(dev)
+            self.ev_host = ev
+            self.event_note = "10^7 events per run (its own seeded draw, Morton order)"
+        elif name == "multirun":
+            # configs[3]: the 120-run x 24-op CORELLI scan strong-scaled over the ranks (contiguous
+            # run blocks, Algorithm 1's range(rank, size), P:76) with one collective
+            wl = synth.make_workload("multirun")
+            from paper_conf_sc_hahnfgmmshvvs24_b200 import plan_shards
+            plan = plan_shards(world, rank, wl.nruns, wl.npix, wl.events_per_run)
+            self.runs = plan.runs
+            self.scaling = "strong"
+            ev = synth.events_for_run(wl, self.runs[0])
+            self.ev_dev = torch.from_numpy(ev).to(dev)
+            self.ev_host = None
+            self.event_note = ("10^7 events per run; each rank bins one seeded 10^7-event draw (its first "
+                               "run's) once per run it owns (BinMD cost does not depend on the run index)")
+        elif name == "topaz":
+            # configs[2] at nops ops (default 48, m-3m); weak scaling like corelli
+            wl = synth.make_workload("topaz", nops=nops or 48)
+            if world > 1:
+                wl.R = np.stack([synth.rot_y(33.0 + 3.0 * r) for r in range(world)])
+                wl.charge = np.ones(world)
+            self.runs = [rank if world > 1 else 0]
+            self.scaling = "weak"
+            ev = synth.events_for_run(wl, self.runs[0], n=10_000_000)
+            ev_d = torch.from_numpy(ev).to(dev)
+            self.ev_dev = torch.cat([ev_d] * 10)  # 10^8 events: ten copies of one Morton-ordered draw
+            del ev_d
+            self.ev_host = None
+            self.event_note = "10^8 events per run = ten copies of one seeded Morton-ordered 10^7-event draw"
+        else:
+            raise ValueError(name)
+        self.wl = wl
+        self.m = m
+        g = m.mdnorm_create_grid(local_rank, wl.lo, wl.hi, wl.nbins, wl.W, m.MDN_ACC_F64)
+        m.mdnorm_set_instrument(g, wl.pix_dir, wl.solid)
+        m.mdnorm_set_flux(g, wl.flux_k, wl.flux_F)
+        self.g = g
+        self.packed = m.packed_histograms(g)
+        self.xs_dev = torch.empty(g.nbins_total, dtype=torch.float64, device=dev)
+        self.traj_rank = len(self.runs) * wl.npix * wl.nops
+        self.events_rank = len(self.runs) * self.ev_dev.shape[0]
+        self.traj_total = (wl.nruns if name == "multirun" else world) * wl.npix * wl.nops
+        self.events_total = self.events_rank * (1 if name == "multirun" else world) if name != "multirun" \
+            else wl.nruns * self.ev_dev.shape[0]
+
+    def step(self, ph=None, events=None):
+        """mdnorm_reset + MDNorm of this rank's runs + BinMD of their events (+ one reduce of
+        [norm | binmd] when N > 1) + the cross-section on rank 0.  ph: five CUDA events recorded
+        between the phases (the phase pass), or None (the headline pass)."""
+        m, wl, g = self.m, self.wl, self.g
         rec = (lambda i: ph[i].record()) if ph is not None else (lambda i: None)
         m.mdnorm_reset(g)
         rec(0)
-        m.mdnorm_accumulate(g, wl.UB, R, wl.ops, wl.k_min, wl.k_max, c)
+        if len(self.runs) == 1:
+            r = self.runs[0]
+            m.mdnorm_accumulate(g, wl.UB, wl.R[r], wl.ops, wl.k_min, wl.k_max, float(wl.charge[r]))
+        else:
+            m.mdnorm_accumulate_runs(g, wl.UB, wl.R[self.runs], wl.charge[self.runs], wl.ops, wl.k_min, wl.k_max)
         rec(1)
-        m.binmd_accumulate(g, wl.UB, wl.ops, ev_dev)
+        for _ in self.runs:
+            m.binmd_accumulate(g, wl.UB, wl.ops, self.ev_dev if events is None else events)
         rec(2)
-        if world > 1:
-            m.reduce_packed(packed, dst=0)
+        if self.world > 1:
+            m.reduce_packed(self.packed, dst=0, nbins=g.nbins_total)
         rec(3)
-        if rank == 0:
-            m.mdnorm_cross_section(g, xs_dev)
+        if self.rank == 0:
+            m.mdnorm_cross_section(g, self.xs_dev if events is None else self.xs_out)
         rec(4)
 
+    def config(self):
+        wl = self.wl
+        d = {"workload": {"corelli": "corelli (BASELINE.json configs[1])",
+                          "multirun": "corelli multi-run rotation scan (BASELINE.json configs[3])",
+                          "topaz": f"topaz, {wl.nops} ops (BASELINE.json configs[2])"}[self.name],
+             "pixels": wl.npix, "ops": wl.nops, "runs_total": wl.nruns if self.name == "multirun" else self.world,
+             "runs_per_gpu": len(self.runs), "trajectories_per_gpu": self.traj_rank,
+             "events_per_gpu": self.events_rank, "events": self.event_note,
+             "grid": [int(x) for x in wl.nbins],
+             "grid_extent": [[float(a), float(b)] for a, b in zip(wl.lo, wl.hi)],
+             "event_order": "coarse-Q Morton (MDBox/SaveMD order)", "acc": "fp64",
+             "l2": "flushed between timed steps (256 MiB device write)"}
+        if self.world > 1:
+            d["parallelism"] = (f"dp{self.world}: " + ("rank r = run r" if self.scaling == "weak"
+                                                        else "contiguous run blocks per rank")
+                                + "; one NCCL reduce of [norm | binmd] to rank 0")
+        else:
+            d["parallelism"] = "single GPU"
+        return d
+
+
+def time_case(case, args, steps, warmup, torch, dist, dev, flush, want_stats=True):
+    """Warm-up, then a headline pass (step events only) and a phase pass (events between the
+    kernels); both bracketed by barrier + synchronize; max over ranks of the summed step time."""
+    m, world, local_rank = case.m, case.world, torch.cuda.current_device()
     mk = lambda: [torch.cuda.Event(enable_timing=True) for _ in range(5)]  # noqa: E731
-    # work counters from one untimed step (tracing; counted kernels are a separate variant)
-    m.mdnorm_stats(g, 1, read=False)
-    step(mk())
-    stats = m.mdnorm_stats(g, 0)
-    for _ in range(args.warmup):
-        step(mk())
+    stats = None
+    if want_stats:
+        m.mdnorm_stats(case.g, 1, read=False)
+        case.step(mk())
+        stats = m.mdnorm_stats(case.g, 0)
+    for _ in range(warmup):
+        case.step(mk())
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
-    starts = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
-    stops = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
-    phases = [mk() for _ in range(args.steps)]
-    # Two timed passes of K steps each, both bracketed by barrier + synchronize: the headline pass
-    # (step events only) gives `value`; the phase pass records an event between the kernels of
-    # every step and gives the per-kernel times of the roofline.
+    starts = [torch.cuda.Event(enable_timing=True) for _ in range(steps)]
+    stops = [torch.cuda.Event(enable_timing=True) for _ in range(steps)]
+    phases = [mk() for _ in range(steps)]
     with ClockSampler(local_rank) as clk:
-        for k in range(args.steps):
+        for k in range(steps):
             flush.zero_()  # L2 flush (outside the timed events)
             starts[k].record()
-            step(None)
+            case.step(None)
             stops[k].record()
         torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     with ClockSampler(local_rank) as clk_ph:
-        for k in range(args.steps):
+        for k in range(steps):
             flush.zero_()
-            step(phases[k])
+            case.step(phases[k])
         torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
@@ -355,53 +448,79 @@ def run_ours(args, rank, world, local_rank):
     total_ms = float(total_ms.item())
     ph_ms = {name: statistics.mean(p[i].elapsed_time(p[i + 1]) for p in phases)
              for i, name in enumerate(["mdnorm", "binmd", "reduce", "xs"])}
+    return {"ms_per_step": total_ms / steps, "phase_ms": ph_ms, "stats": stats, "clocks": clk.summary(),
+            "clocks_phase": clk_ph.summary(), "step_ms_rank0": step_ms}
+
+
+def case_summary(case, t, steps, warmup):
+    ms = t["ms_per_step"]
+    st = t["stats"] or {}
+    out = {"metric": METRIC, "value": case.traj_total / (ms / 1e3), "unit": UNIT, "n_gpus": case.world,
+           "steps": steps, "warmup": warmup, "ms_per_step": ms, "scaling": case.scaling,
+           "config": case.config(), "clocks": t["clocks"],
+           "binmd_events_per_s": case.events_total / (ms / 1e3),
+           "phase_ms": t["phase_ms"],
+           "mdnorm_kernel_traj_per_s": case.traj_rank / (t["phase_ms"]["mdnorm"] / 1e3),
+           "binmd_kernel_events_per_s": case.events_rank / (t["phase_ms"]["binmd"] / 1e3),
+           "work_counts_rank0": st}
+    if st.get("segments"):
+        out["mdnorm_segments_per_s"] = st["segments"] / (t["phase_ms"]["mdnorm"] / 1e3)
+    return out
+
+
+def run_ours(args, rank, world, local_rank):
+    import torch
+    import torch.distributed as dist
+    import synth
+    import paper_conf_sc_hahnfgmmshvvs24_b200 as m
+    from paper_conf_sc_hahnfgmmshvvs24_b200 import build
+
+    build.build()
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    case = Case(m, torch, synth, args.config, world, rank, local_rank, dev, nops=args.nops)
+    wl, g = case.wl, case.g
+    t = time_case(case, args, args.steps, args.warmup, torch, dist, dev, flush)
+    stats, ph_ms = t["stats"], t["phase_ms"]
 
     # ---------------- end to end through the C ABI with HOST buffers (pinned), copies inside
-    ev_pin = torch.from_numpy(ev).pin_memory()
-    xs_pin = torch.empty(g.nbins_total, dtype=torch.float64).pin_memory()
-
-    def step_e2e():
-        m.mdnorm_reset(g)
-        m.mdnorm_accumulate(g, wl.UB, R, wl.ops, wl.k_min, wl.k_max, c)
-        m.binmd_accumulate(g, wl.UB, wl.ops, ev_pin)          # chunked H2D overlapped with scatter
-        if world > 1:
-            m.reduce_packed(packed, dst=0)
-        if rank == 0:
-            m.mdnorm_cross_section(g, xs_pin)                   # D2H + synchronise
-
-    for _ in range(2):
-        step_e2e()
-    torch.cuda.synchronize()
-    if world > 1:
-        dist.barrier()
-    e_starts = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
-    e_stops = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
-    with ClockSampler(local_rank) as clk_e2e:
-        for k in range(args.steps):
-            flush.zero_()
-            e_starts[k].record()
-            step_e2e()
-            e_stops[k].record()
+    e2e = None
+    if case.ev_host is not None:
+        ev_pin = torch.from_numpy(case.ev_host).pin_memory()
+        xs_pin = torch.empty(g.nbins_total, dtype=torch.float64).pin_memory()
+        case.xs_out = xs_pin
+        for _ in range(2):
+            case.step(None, events=ev_pin)
         torch.cuda.synchronize()
-    e2e_ms = torch.tensor([sum(a.elapsed_time(b) for a, b in zip(e_starts, e_stops))], dtype=torch.float64,
-                          device=dev)
-    if world > 1:
-        dist.all_reduce(e2e_ms, op=dist.ReduceOp.MAX)
-    e2e_ms = float(e2e_ms.item())
+        if world > 1:
+            dist.barrier()
+        e_starts = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+        e_stops = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+        with ClockSampler(local_rank) as clk_e2e:
+            for k in range(args.steps):
+                flush.zero_()
+                e_starts[k].record()
+                case.step(None, events=ev_pin)  # chunked H2D overlapped with BinMD; D2H xs + sync
+                e_stops[k].record()
+            torch.cuda.synchronize()
+        e2e_ms = torch.tensor([sum(a.elapsed_time(b) for a, b in zip(e_starts, e_stops))], dtype=torch.float64,
+                              device=dev)
+        if world > 1:
+            dist.all_reduce(e2e_ms, op=dist.ReduceOp.MAX)
+        e2e_ms = float(e2e_ms.item())
+        if rank == 0:
+            assert np.isfinite(xs_pin.numpy()).sum() > 1000, "cross-section has too few finite bins"
+        e2e = {"value": case.traj_total / (e2e_ms / args.steps / 1e3), "unit": UNIT,
+               "ms_per_step": e2e_ms / args.steps,
+               "h2d_bytes_per_step": int(case.ev_host.nbytes) * world,
+               "d2h_bytes_per_step": 8 * g.nbins_total,
+               "clocks": clk_e2e.summary(),
+               "path": "C ABI with pinned host events (chunked H2D overlapped with BinMD) and host xs"}
 
-    # sanity: the result of the last step is a real cross-section
-    if rank == 0:
-        xs_np = xs_pin.numpy()
-        finite = np.isfinite(xs_np)
-        assert finite.sum() > 1000, "cross-section has too few finite bins"
-
-    traj_total = wl.npix * wl.nops * world
-    ev_total = len(ev) * world
-    ms_per_step = total_ms / args.steps
-    value = traj_total / (ms_per_step / 1e3)
-
+    ms_per_step = t["ms_per_step"]
+    value = case.traj_total / (ms_per_step / 1e3)
     peaks, peaks_src = measured_peaks()
-    clocks = clk.summary()
     sm_max = float(peaks.get("sm_max_mhz", 1965.0))
     fp64_peak = fp64_peak_tops(sm_max)
     hbm = float(peaks["hbm_gbs"])
@@ -409,18 +528,18 @@ def run_ours(args, rank, world, local_rank):
     kernels = {}
     md_ops = OPS_PER_TRAJ * stats["trajectories"] + OPS_PER_HIT * stats["hit_trajectories"] + \
         OPS_PER_SEG * stats["segments"]
-    t = ph_ms["mdnorm"] / 1e3
+    tm = ph_ms["mdnorm"] / 1e3
     md_traffic = None
     if "mdnorm_cull_kernel" in traffic and "mdnorm_walk_kernel" in traffic:
         md_traffic = traffic["mdnorm_cull_kernel"] + traffic["mdnorm_walk_kernel"]
-    alu = {"bound": "alu", "achieved": md_ops / t / 1e12, "peak": fp64_peak, "unit": "TFLOP/s",
-           "frac": md_ops / t / 1e12 / fp64_peak,
+    alu = {"bound": "alu", "achieved": md_ops / tm / 1e12, "peak": fp64_peak, "unit": "TFLOP/s",
+           "frac": md_ops / tm / 1e12 / fp64_peak,
            "peak_note": f"fp64 non-fused ops at {sm_max:.0f} MHz (148 SM x 64 lanes), DESIGN.md §4"}
     aroof, aroof_src = atomic_roof()
     if aroof:
         # one fp64 red.add per segment (M7): the tighter of the two roofs
-        kernels["mdnorm"] = {"bound": "atomic", "achieved": stats["segments"] / t / 1e9, "peak": aroof / 1e9,
-                             "unit": "Gatomic/s", "frac": stats["segments"] / t / aroof,
+        kernels["mdnorm"] = {"bound": "atomic", "achieved": stats["segments"] / tm / 1e9, "peak": aroof / 1e9,
+                             "unit": "Gatomic/s", "frac": stats["segments"] / tm / aroof,
                              "peak_source": f"measured: {aroof_src} (fp64 red.global.add, L2-resident bins)",
                              "alu": alu}
     else:
@@ -428,55 +547,87 @@ def run_ours(args, rank, world, local_rank):
     kernels["mdnorm"].update({"kernels": "mdnorm_cull_kernel + mdnorm_walk_kernel", "traffic": md_traffic,
                               "ms": ph_ms["mdnorm"], "ops_per_launch": md_ops,
                               "segments_per_launch": stats["segments"]})
-    t = ph_ms["binmd"] / 1e3
-    bm_bytes = BYTES_PER_EVENT * len(ev)
-    kernels["binmd_kernel"] = {"bound": "hbm", "achieved": bm_bytes / t / 1e9, "peak": hbm,
-                               "unit": "GB/s", "frac": bm_bytes / t / 1e9 / hbm,
+    tb = ph_ms["binmd"] / 1e3
+    bm_bytes = BYTES_PER_EVENT * case.events_rank
+    kernels["binmd_kernel"] = {"bound": "hbm", "achieved": bm_bytes / tb / 1e9, "peak": hbm,
+                               "unit": "GB/s", "frac": bm_bytes / tb / 1e9 / hbm,
                                "traffic": traffic.get("binmd_kernel"), "ms": ph_ms["binmd"],
-                               "bytes_per_launch": bm_bytes}
-    t = ph_ms["xs"] / 1e3
-    if rank == 0 and t > 0:
+                               "bytes_per_launch": bm_bytes,
+                               "peak_source": f"{peaks_src}: MEASURED_PEAKS.json hbm_gbs"}
+    tx = ph_ms["xs"] / 1e3
+    if rank == 0 and tx > 0:
         xs_bytes = 24 * g.nbins_total
-        kernels["xs_kernel"] = {"bound": "hbm", "achieved": xs_bytes / t / 1e9, "peak": hbm, "unit": "GB/s",
-                                "frac": xs_bytes / t / 1e9 / hbm, "ms": ph_ms["xs"]}
+        kernels["xs_kernel"] = {"bound": "hbm", "achieved": xs_bytes / tx / 1e9, "peak": hbm, "unit": "GB/s",
+                                "frac": xs_bytes / tx / 1e9 / hbm, "ms": ph_ms["xs"]}
     dom = max(("mdnorm", "binmd_kernel"), key=lambda k: kernels[k]["ms"])
     roof = {k: kernels[dom][k] for k in ("bound", "achieved", "peak", "unit", "frac", "traffic")}
     roof["kernel"] = kernels[dom].get("kernels", dom)
     roof["peak_source"] = kernels[dom].get("peak_source", f"{peaks_src}: MEASURED_PEAKS.json hbm_gbs")
 
+    # our kernels per step: cull + walk per slab of every launch block (16 runs per block), one
+    # binmd per run, the divide on rank 0
+    blocks = -(-len(case.runs) // 16)
+    slabs = m.mdnorm_debug_last_launch(case.g)["slabs"]
+    launches_per_step = 2 * slabs * blocks + len(case.runs) + (1 if rank == 0 else 0)
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
-        "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
-        "vs_baseline": None, "dtype": "f64", "data": "synthetic (seeded, SURVEY.md §8(d) CORELLI recipe)",
-        "config": config_dict(wl, world),
-        "secondary": {"binmd_events_per_s": ev_total / (ms_per_step / 1e3),
-                      "mdnorm_kernel_traj_per_s": wl.npix * wl.nops / (ph_ms["mdnorm"] / 1e3),
-                      "binmd_kernel_events_per_s": len(ev) / (ph_ms["binmd"] / 1e3),
+        "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": case.scaling,
+        "vs_baseline": None, "dtype": "f64", "data": "synthetic (seeded, SURVEY.md §8(d) recipe)",
+        "config": case.config(),
+        "secondary": {"binmd_events_per_s": case.events_total / (ms_per_step / 1e3),
+                      "mdnorm_kernel_traj_per_s": case.traj_rank / (ph_ms["mdnorm"] / 1e3),
+                      "binmd_kernel_events_per_s": case.events_rank / (ph_ms["binmd"] / 1e3),
                       "mdnorm_segments_per_s": stats["segments"] / (ph_ms["mdnorm"] / 1e3),
                       "phase_ms": ph_ms, "work_counts_rank0": stats,
-                      "phase_pass": {"steps": args.steps, "clocks": clk_ph.summary(),
+                      "phase_pass": {"steps": args.steps, "clocks": t["clocks_phase"],
                                      "note": "per-kernel times (phase_ms, roofline) come from a second timed pass "
                                              "with an event between kernels; value comes from the pass without"}},
-        "clocks": clocks,
-        "e2e": {"value": traj_total / (e2e_ms / args.steps / 1e3), "unit": UNIT,
-                "ms_per_step": e2e_ms / args.steps,
-                "h2d_bytes_per_step": int(ev.nbytes) * world,
-                "d2h_bytes_per_step": 8 * g.nbins_total,
-                "clocks": clk_e2e.summary(),
-                "path": "C ABI with pinned host events (chunked H2D overlapped with BinMD) and host xs"},
-        "gpu_launches": args.steps * (3 + (1 if rank == 0 else 0)),  # cull, walk, binmd (+ xs)
+        "clocks": t["clocks"],
+        "gpu_launches": args.steps * launches_per_step,  # cull + walk per slab, binmd per run, xs on rank 0
         "roofline": roof,
         "kernels": kernels,
     }
+    if e2e:
+        line["e2e"] = e2e
+    case.g.close()
+    del case
+    torch.cuda.empty_cache()
+    # ---------------- the other BASELINE configs, measured in the same invocation
+    extras = {}
+    for name in [x for x in args.extra_configs.split(",") if x and x != args.config]:
+        if name == "topaz" and world > 1 and not args.extra_weak:
+            continue
+        c2 = Case(m, torch, synth, name, world, rank, local_rank, dev, nops=None)
+        steps2 = max(3, min(args.steps, 5))
+        t2 = time_case(c2, args, steps2, 3, torch, dist, dev, flush)
+        extras[name] = case_summary(c2, t2, steps2, 3)
+        c2.g.close()
+        del c2
+        torch.cuda.empty_cache()
+    if extras:
+        line["configs"] = extras
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        line["cpu_baseline"] = cpu_baseline(wl, ev, args.cpu_stride)
+        wl0 = synth.make_workload("corelli")
+        line["cpu_baseline"] = cpu_baseline(wl0, synth.events_for_run(wl0, 0), args.cpu_stride)
     if rank == 0:
         print(json.dumps(line), flush=True)
         if args.json_out:
             with open(args.json_out, "w") as f:
                 json.dump(line, f, indent=1)
-    g.close()
     return 0
+
+
+def spawn_ranks(args) -> int:
+    """`bench.py --gpus N` outside torchrun: launch N ranks with torch.distributed.run on
+    127.0.0.1 (one process per GPU) and return their exit status."""
+    import socket
+    import subprocess
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.run(cmd).returncode
 
 
 def main():
@@ -485,18 +636,29 @@ def main():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--config", choices=["corelli", "multirun", "topaz"], default="corelli",
+                    help="headline workload (default: BASELINE.json configs[1])")
+    ap.add_argument("--nops", type=int, default=None, help="symmetry ops of the topaz config (default 48)")
+    ap.add_argument("--extra-configs", default="multirun,topaz",
+                    help="other BASELINE configs timed in the same run and reported under 'configs' ('' = none)")
+    ap.add_argument("--extra-weak", action="store_true", help="also time the topaz extra at N > 1")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-stride", type=int, default=1, help="oracle sample: every n-th pixel and event")
     ap.add_argument("--ref-stride", type=int, default=1, help="--impl reference per-step sample stride")
     ap.add_argument("--json-out", default=None)
-    ap.add_argument("--dist-backend", default="nccl",
-                    help="nccl (production); gloo + MDN_BENCH_SHARED_GPU=1 exercises the N>1 code "
-                         "path with every rank on GPU 0 (tests only; not a performance number)")
     args = ap.parse_args()
-    world = int(os.environ.get("WORLD_SIZE", "1"))
+    if args.warmup < 3 and args.impl == "ours":
+        ap.error("at least 3 warm-up steps")
+    world_env = os.environ.get("WORLD_SIZE")
+    if world_env is None and args.gpus > 1:
+        return spawn_ranks(args)
+    world = int(world_env or "1")
+    if world != args.gpus:
+        ap.error(f"--gpus {args.gpus} but WORLD_SIZE={world}")
     rank = int(os.environ.get("RANK", "0"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
-    if os.environ.get("MDN_BENCH_SHARED_GPU") == "1":
+    shared = os.environ.get("MDN_BENCH_SHARED_GPU") == "1"
+    if shared:  # tests only: every rank on GPU 0 (NCCL refuses two ranks on one GPU: gloo)
         local_rank = 0
     if args.impl == "reference":
         return run_reference(args, rank, world)
@@ -504,10 +666,10 @@ def main():
         import torch
         import torch.distributed as dist
         torch.cuda.set_device(local_rank)
-        if args.dist_backend == "nccl":
-            dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        if shared:
+            dist.init_process_group("gloo")
         else:
-            dist.init_process_group(args.dist_backend)
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
     try:
         return run_ours(args, rank, world, local_rank)
     finally:

@@ -255,7 +255,9 @@ def test_topaz_pixel_subsample_parity(mdn, nops):
 
 def test_topaz_full_size_properties(mdn):
     """Full TOPAZ-shaped launch (1.64M px x 8 ops): linearity over pixel shards (a property that
-    holds at any size) and the shard with stride 4001 against the oracle."""
+    holds at any size: four interleaved shards sum to the one launch) and 2M of its events
+    through BinMD against the oracle.  The full launch itself is compared with the oracle bin by
+    bin in tests/test_gpu_fullsize.py::test_topaz_8ops_full_pixels."""
     wl = synth.make_workload("topaz", nops=8)
     g = make_grid(mdn, wl)
     mdn.mdnorm_accumulate(g, wl.UB, wl.R[0], wl.ops, wl.k_min, wl.k_max, 1.0)
