@@ -52,6 +52,14 @@ struct mdn_grid {
   cudaEvent_t ev_ready[2] = {nullptr, nullptr};
   cudaEvent_t ev_free[2] = {nullptr, nullptr};
   cudaEvent_t ev_epoch = nullptr;  // recorded by mdnorm_reset: host-event copies start after it
+  // BinMD decision tables (B0, launch_binmd_plan): two buffers used in turn; the plan of a call
+  // runs on plan_stream (it depends on no device data, so it overlaps the MDNorm kernels before
+  // it) and the BinMD kernels wait for it
+  void* d_btab[2] = {nullptr, nullptr};
+  int btab_i = 0;
+  cudaStream_t plan_stream = nullptr;
+  cudaEvent_t ev_tab_ready[2] = {nullptr, nullptr};
+  cudaEvent_t ev_tab_free[2] = {nullptr, nullptr};
 };
 
 namespace {
@@ -294,7 +302,7 @@ mdn::BinParams bin_params(mdn_grid* g, const float* ev, int64_t n, const EvLayou
 // Run the BinMD kernel over host events through a two-slot staging ring: the H2D copy of chunk
 // c+1 (copy stream) overlaps the scatter of chunk c (caller's stream).
 mdn_status binmd_host_stream(mdn_grid* g, const MatBlock& mb, int64_t nevents, const float* events,
-                             const EvLayout& L, cudaStream_t s) {
+                             const EvLayout& L, cudaStream_t s, const void* tables) {
   const int64_t stride = L.stride;
   const int64_t chunk = std::max<int64_t>(1, (int64_t)(64ll << 20) / (int64_t)(4 * stride));  // 64 MB
   const size_t need = (size_t)(chunk * stride);
@@ -334,23 +342,58 @@ mdn_status binmd_host_stream(mdn_grid* g, const MatBlock& mb, int64_t nevents, c
                              cudaMemcpyHostToDevice, g->copy_stream), "H2D events");
     MDN_CUDA(cudaEventRecord(g->ev_ready[slot], g->copy_stream), "event record");
     MDN_CUDA(cudaStreamWaitEvent(s, g->ev_ready[slot], 0), "wait");
-    MDN_CUDA(mdn::launch_binmd(bin_params(g, g->d_stage[slot], n, L), mb, g->num_sms, s), "binmd kernel");
+    mdn::BinParams p = bin_params(g, g->d_stage[slot], n, L);
+    p.tables = tables;
+    MDN_CUDA(mdn::launch_binmd(p, mb, g->num_sms, s), "binmd kernel");
     g->path[1] = mdn::last_binmd_path();
     MDN_CUDA(cudaEventRecord(g->ev_free[slot], s), "event record");
   }
   return MDN_OK;
 }
 
+// B0 of one BinMD call: the plan kernel on plan_stream into the next table buffer, ordered after
+// the last kernels that read that buffer; returns the buffer (the caller's kernels wait on
+// ev_tab_ready and record ev_tab_free after them).
+mdn_status binmd_plan(mdn_grid* g, const MatBlock& mb, const EvLayout& L, cudaStream_t s, int* slot) {
+  if (!g->plan_stream) {
+    MDN_CUDA(cudaStreamCreateWithFlags(&g->plan_stream, cudaStreamNonBlocking), "plan stream");
+    for (int i = 0; i < 2; ++i) {
+      MDN_CUDA(cudaEventCreateWithFlags(&g->ev_tab_ready[i], cudaEventDisableTiming), "event");
+      MDN_CUDA(cudaEventCreateWithFlags(&g->ev_tab_free[i], cudaEventDisableTiming), "event");
+    }
+  }
+  const int i = g->btab_i ^ 1;
+  if (!g->d_btab[i]) MDN_CUDA(cudaMalloc(&g->d_btab[i], mdn::binmd_tables_bytes()), "binmd tables");
+
+  // the plan runs after the caller's work up to its last reset (the start of its accumulation
+  // epoch, as for host-event copies) and after the last kernels that read this buffer
+  if (g->ev_epoch) MDN_CUDA(cudaStreamWaitEvent(g->plan_stream, g->ev_epoch, 0), "wait");
+  MDN_CUDA(cudaStreamWaitEvent(g->plan_stream, g->ev_tab_free[i], 0), "wait");
+  MDN_CUDA(mdn::launch_binmd_plan(bin_params(g, nullptr, 0, L), mb, g->d_btab[i], g->plan_stream), "binmd plan");
+  MDN_CUDA(cudaEventRecord(g->ev_tab_ready[i], g->plan_stream), "event record");
+  MDN_CUDA(cudaStreamWaitEvent(s, g->ev_tab_ready[i], 0), "wait");
+  g->btab_i = i;
+  *slot = i;
+  return MDN_OK;
+}
+
 mdn_status binmd_run(mdn_grid* g, const MatBlock& mb, int64_t nevents, const float* events, const EvLayout& L,
                      cudaStream_t s) {
   if (nevents == 0) return ok();
+  int slot = 0;
+  mdn_status st = binmd_plan(g, mb, L, s, &slot);
+  if (st != MDN_OK) return st;
   if (is_device_ptr(events)) {
-    MDN_CUDA(mdn::launch_binmd(bin_params(g, events, nevents, L), mb, g->num_sms, s), "binmd kernel");
+    mdn::BinParams p = bin_params(g, events, nevents, L);
+    p.tables = g->d_btab[slot];
+    MDN_CUDA(mdn::launch_binmd(p, mb, g->num_sms, s), "binmd kernel");
     g->path[1] = mdn::last_binmd_path();
-    return ok();
+  } else {
+    st = binmd_host_stream(g, mb, nevents, events, L, s, g->d_btab[slot]);
+    if (st != MDN_OK) return st;
   }
-  mdn_status st = binmd_host_stream(g, mb, nevents, events, L, s);
-  return st == MDN_OK ? ok() : st;
+  MDN_CUDA(cudaEventRecord(g->ev_tab_free[slot], s), "event record");
+  return ok();
 }
 
 }  // namespace
@@ -430,6 +473,12 @@ mdn_status mdnorm_destroy(mdn_grid* g) {
   }
   if (g->ev_epoch) cudaEventDestroy(g->ev_epoch);
   if (g->copy_stream) cudaStreamDestroy(g->copy_stream);
+  for (int i = 0; i < 2; ++i) {
+    cudaFree(g->d_btab[i]);
+    if (g->ev_tab_ready[i]) cudaEventDestroy(g->ev_tab_ready[i]);
+    if (g->ev_tab_free[i]) cudaEventDestroy(g->ev_tab_free[i]);
+  }
+  if (g->plan_stream) cudaStreamDestroy(g->plan_stream);
   delete g;
   cudaGetLastError();
   return ok();

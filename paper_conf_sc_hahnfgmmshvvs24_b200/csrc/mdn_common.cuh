@@ -54,10 +54,20 @@ __device__ __forceinline__ void flush_counter(unsigned long long* dst, unsigned 
 // measured slower on this B200 -- BinMD 2x on the Morton-ordered CORELLI events, 1.8x on TOPAZ
 // 48 ops, 1.6x into a private shared-memory grid; the walk 1.4-1.75x -- so every
 // contribution is its own reduction.
+// The global fp64 form is an explicit fire-and-forget reduction (red.global.add.f64): the
+// compiler otherwise emits an atomic with a (discarded) return in code that also holds
+// acquire/release operations, which waits for the L2 round trip.
+__device__ __forceinline__ void red_add(double* p, double v) {
+  asm volatile("red.relaxed.gpu.global.add.f64 [%0], %1;" ::"l"(p), "d"(v) : "memory");
+}
 template <typename T>
 __device__ __forceinline__ void hist_add(T* h, T* h2, int b, T v, T v2, bool two) {
   atomicAdd(h + b, v);
   if (two) atomicAdd(h2 + b, v2);
+}
+__device__ __forceinline__ void hist_add(double* h, double* h2, int b, double v, double v2, bool two) {
+  red_add(h + b, v);
+  if (two) red_add(h2 + b, v2);
 }
 
 // Zero the CTA's private histogram (before the kernel's first __syncthreads).

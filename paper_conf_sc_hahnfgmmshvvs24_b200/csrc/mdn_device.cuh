@@ -86,11 +86,15 @@ __device__ __forceinline__ bool inv3_scaled(const double* C, double scale, doubl
   bool fast = recip_range(det);
 #pragma unroll
   for (int i = 0; i < 9; ++i) fast = fast && recip_range(cof[i]);
+  if (fast) {
 #pragma unroll
-  for (int i = 0; i < 3; ++i)
+    for (int i = 0; i < 3; ++i)
 #pragma unroll
-    for (int j = 0; j < 3; ++j)
-      out[3 * i + j] = dmul(fast ? div_rn_recip(cof[3 * j + i], det, y) : ddiv(cof[3 * j + i], det), scale);
+      for (int j = 0; j < 3; ++j) out[3 * i + j] = dmul(div_rn_recip(cof[3 * j + i], det, y), scale);
+  } else {
+    for (int i = 0; i < 3; ++i)
+      for (int j = 0; j < 3; ++j) out[3 * i + j] = dmul(ddiv(cof[3 * j + i], det), scale);
+  }
   return true;
 }
 

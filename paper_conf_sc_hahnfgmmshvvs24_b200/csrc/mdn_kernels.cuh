@@ -95,6 +95,7 @@ struct BinParams {
   double* binmd;           // fp64 histogram (nbins)
   double* err2;            // fp64 error-squared histogram (nbins), used when col_e >= 0
   unsigned long long* stats;  // nullptr, or [.., .., .., .., pairs, inside] (+= per launch)
+  const void* tables;      // the launch's BinTables in global memory (launch_binmd_plan)
 };
 
 // launchers (return the launch's cudaError_t)
@@ -106,6 +107,10 @@ cudaError_t launch_mdnorm(const MdnParams& p, const MatBlock& mb, int num_sms, c
 // per-CTA blocks): the walk's large-launch regime (tests assert they cover it).
 uint32_t walk_big_claim_threshold(bool d3, int num_sms);
 cudaError_t launch_binmd(const BinParams& p, const MatBlock& mb, int num_sms, cudaStream_t s);
+// B0 for one BinMD launch: compose N_s and build the decision tables into `tables` (device memory
+// of binmd_tables_bytes()), one CTA; binmd_kernel reads them (BinParams::tables).
+size_t binmd_tables_bytes();
+cudaError_t launch_binmd_plan(const BinParams& p, const MatBlock& mb, void* tables, cudaStream_t s);
 // Accumulation path chosen for the last launch_mdnorm / launch_binmd on this thread (tracing and
 // tests): 0 = global fp64 red.add, 1 = shared-memory fp64 partials, 2 = shared-memory fp32 partials.
 int last_mdnorm_path();
