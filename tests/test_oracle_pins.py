@@ -475,3 +475,62 @@ def test_error_histogram_pins(orc):
     assert np.array_equal(np.isnan(s1), np.isnan(x1))
     np.testing.assert_allclose(x2[ok], x1[ok], rtol=1e-15)
     np.testing.assert_allclose(s2[ok], s1[ok] / math.sqrt(2.0), rtol=1e-15)
+
+
+# ----------------------------------------------------------------------------- second pins (r02)
+
+
+def test_segments_have_positive_length(orc):
+    """Reading #7 (skip only k2 <= k1): on a diagonal trajectory whose H and K crossings
+    coincide at every grid corner (v = (a, a, 0), square bins), L has tied entries; the oracle
+    keeps exactly one segment per distinct pair of consecutive values, every one of positive
+    value under a flux of positive density -- n_seg = distinct crossings + 1 (closed form)."""
+    a = 0.37
+    M = np.diag([a, a, 0.0]) / a  # v = M q; q = z - d with d chosen so q = (1, 1, 0) * s
+    # pixel direction with q = z - d = (c, c, 0): d = (-c, -c, 1); not unit -- the oracle takes d as given
+    c = 0.8
+    d = np.array([-c, -c, 1.0])
+    lo, hi, n = [0.0, 0.0, -1.0], [4.0, 4.0, 1.0], [8, 8, 1]
+    grid = orc.Grid(lo, hi, n)
+    fk, fF = np.array([0.1, 50.0]), np.array([0.0, 49.9])  # uniform density 1
+    kmin, kmax = 0.3, 4.7
+    nc, ns, bins, vals = orc.mdnorm_trajectory(grid, d, 1.0, fk, fF, M, 1.0, kmin, kmax)
+    # x(k) = k c (1, 1, 0): inside for k c in [0, 4); every plane j * 0.5 crosses both axes at once
+    kin, kout = kmin, min(kmax, 4.0 / c)
+    distinct = [j * 0.5 / c for j in range(1, 8) if kin < j * 0.5 / c < kout]
+    assert ns == len(distinct) + 1
+    assert np.all(vals > 0)
+    assert np.isclose(vals.sum(), kout - kin, rtol=1e-13)
+
+
+def test_rotated_goniometer_bragg_trajectory(orc):
+    """Second pin on the composition order M = (R UB S W)^-1 / 2 pi (reading #2) through the
+    trajectory geometry: for a reflection h, the physics forward model gives Q_lab = R 2 pi UB h;
+    the elastic pixel that sees it is d = z - Q_lab / k* with k* = |Q|^2 / (2 Q_z).  That pixel's
+    trajectory (goniometer R, a narrow k window around k*) must cross the bin of x = W^-1 h."""
+    wl = synth.make_workload("corelli")
+    rng = np.random.default_rng(5)
+    hits = 0
+    for _ in range(40):
+        h = rng.integers(-4, 5, 3).astype(float)
+        h[2] = rng.integers(-2, 3)
+        if not h.any():
+            continue
+        R = synth.rot_y(rng.uniform(0, 360)) @ synth.rot_x(rng.uniform(-20, 20))
+        Q = R @ (2 * math.pi * wl.UB @ h)
+        if Q[2] <= 1e-3:
+            continue  # not reachable in the elastic geometry (needs Q_z > 0)
+        kst = Q @ Q / (2 * Q[2])
+        d = np.array([0.0, 0.0, 1.0]) - Q / kst
+        x = np.linalg.solve(wl.W, h)
+        # grid of 1e-3-wide bins centred on x
+        w = 1e-3
+        lo = x - 1.5 * w
+        grid = orc.Grid(lo, lo + 3 * w, [3, 3, 3])
+        M = orc.compose_mdnorm(R, wl.UB, np.eye(3), wl.W)
+        fk, fF = np.array([0.01, 1e4]), np.array([0.0, 1e4])
+        nc, ns, bins, vals = orc.mdnorm_trajectory(grid, d, 1.0, fk, fF, M, 1.0, kst * (1 - 1e-6), kst * (1 + 1e-6))
+        assert ns > 0, (h, kst)
+        assert 13 in bins.tolist(), (h, bins)  # the centre bin (1, 1, 1) of the 3x3x3 grid
+        hits += 1
+    assert hits >= 10
