@@ -73,7 +73,11 @@ def atomic_roof():
         return None, None
     with open(files[-1]) as f:
         r = json.load(f)
-    return float(r["atomics_per_s"]["corelli_600x600"]["red_f64_random"]), os.path.relpath(files[-1], ROOT)
+    c = r["atomics_per_s"]["corelli_600x600"]
+    src = os.path.relpath(files[-1], ROOT)
+    if "clock" in c:
+        src += f" (SM {c['clock']['sm_mhz_median']} MHz median, throttle reasons {c['clock']['reasons']})"
+    return float(c["red_f64_random"]), src
 
 
 # ----------------------------------------------------------------------------- clocks

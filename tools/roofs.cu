@@ -3,8 +3,11 @@
 // this B200 at whatever clock the driver runs it (no clock changes).  Not part of the product: a
 // standalone executable that prints one JSON object; bench.py / DESIGN.md quote its numbers.
 //
-//   nvcc -O3 -std=c++17 -gencode arch=compute_100a,code=sm_100a -o tools/roofs tools/roofs.cu
+//   nvcc -O3 -std=c++17 -gencode arch=compute_100a,code=sm_100a -o tools/roofs tools/roofs.cu \
+//        -L/usr/local/cuda/lib64/stubs -lnvidia-ml
 //   tools/roofs > profiles/rNN_roofs.json
+// Every case records the SM clock (NVML, sampled every 0.5 ms while it runs: median and
+// minimum) and the OR of the clock-event (throttle) reasons seen, so a roof carries its clock.
 //
 // Cases (all reductions compile to RED.E.ADD: the return value is unused):
 //   red_f64_random  S    fp64 red.global.add to uniformly random bins of an S-byte histogram
@@ -20,8 +23,13 @@
 #include <cstdio>
 #include <cstdint>
 #include <cstdlib>
+#include <algorithm>
+#include <atomic>
 #include <cooperative_groups.h>
 #include <cuda_runtime.h>
+#include <nvml.h>
+#include <thread>
+#include <vector>
 namespace cg = cooperative_groups;
 
 #define CK(x)                                                                         \
@@ -124,26 +132,67 @@ __global__ void fp64_alu(double* out, int iters) {
   if (t == 1234.5) out[0] = t;
 }
 
+// NVML sampler of the SM clock and the clock-event reasons while a case runs.
+struct ClockLog {
+  nvmlDevice_t dev{};
+  bool ok = false;
+  std::vector<unsigned> mhz;
+  unsigned long long reasons = 0;
+  ClockLog() { ok = nvmlInit_v2() == NVML_SUCCESS && nvmlDeviceGetHandleByIndex_v2(0, &dev) == NVML_SUCCESS; }
+  template <class F>
+  void run(F f) {
+    mhz.clear();
+    reasons = 0;
+    std::atomic<bool> stop{false};
+    std::thread th([&] {
+      while (!stop.load() && ok) {
+        unsigned c = 0;
+        unsigned long long r = 0;
+        if (nvmlDeviceGetClockInfo(dev, NVML_CLOCK_SM, &c) == NVML_SUCCESS) mhz.push_back(c);
+        if (nvmlDeviceGetCurrentClocksEventReasons(dev, &r) == NVML_SUCCESS) reasons |= r;
+        std::this_thread::sleep_for(std::chrono::microseconds(500));
+      }
+    });
+    f();
+    stop = true;
+    th.join();
+  }
+  // JSON fragment: "clock": {"sm_mhz_median": M, "sm_mhz_min": m, "samples": n, "reasons": "0x.."}
+  void print(const char* key = "clock") {
+    std::vector<unsigned> v = mhz;
+    std::sort(v.begin(), v.end());
+    // idle (0x1) is expected between the timed repetitions
+    printf("\"%s\": {\"sm_mhz_median\": %u, \"sm_mhz_min\": %u, \"samples\": %zu, \"reasons\": \"0x%llx\"}",
+           key, v.empty() ? 0 : v[v.size() / 2], v.empty() ? 0 : v[0], v.size(), reasons & ~1ull);
+  }
+};
+
 struct Timer {
   cudaEvent_t a, b;
+  ClockLog* log = nullptr;
   Timer() {
     CK(cudaEventCreate(&a));
     CK(cudaEventCreate(&b));
   }
+  // best of `reps` timings, each `inner` back-to-back launches (long enough for clock samples)
   template <class F>
-  float best(F f, int reps = 5) {
+  float best(F f, int reps = 5, int inner = 20) {
     f();
     CK(cudaDeviceSynchronize());
     float best = 1e30f;
-    for (int r = 0; r < reps; ++r) {
-      CK(cudaEventRecord(a));
-      f();
-      CK(cudaEventRecord(b));
-      CK(cudaEventSynchronize(b));
-      float ms;
-      CK(cudaEventElapsedTime(&ms, a, b));
-      if (ms < best) best = ms;
-    }
+    auto body = [&] {
+      for (int r = 0; r < reps; ++r) {
+        CK(cudaEventRecord(a));
+        for (int i = 0; i < inner; ++i) f();
+        CK(cudaEventRecord(b));
+        CK(cudaEventSynchronize(b));
+        float ms;
+        CK(cudaEventElapsedTime(&ms, a, b));
+        if (ms / inner < best) best = ms / inner;
+      }
+    };
+    if (log) log->run(body);
+    else body();
     return best;
   }
 };
@@ -156,6 +205,8 @@ int main() {
   cudaDeviceProp prop;
   CK(cudaGetDeviceProperties(&prop, dev));
   Timer t;
+  ClockLog clog;
+  t.log = &clog;
   const int threads = 512, blocks = nsm * 4;
   const double nthr = (double)threads * blocks;
   printf("{\n \"gpu\": \"%s\", \"sms\": %d, \"l2_bytes\": %d, \"clock_khz_attr\": %d,\n", prop.name, nsm,
@@ -178,14 +229,17 @@ int main() {
     double* hd = static_cast<double*>(h);
     float* hf = static_cast<float*>(h);
     const float ms_r = t.best([&] { red_random<double><<<blocks, threads>>>(hd, nb, iters); });
+    ClockLog cr = clog;
     const float ms_w = t.best([&] { red_walk<<<blocks, threads>>>(hd, c.n0, c.n1, c.n2, iters, 64); });
     const float ms_f = t.best([&] { red_random<float><<<blocks, threads>>>(hf, nb, iters); });
     CK(cudaGetLastError());
     const double n = nthr * iters;
     printf("  \"%s\": {\"bins\": %u, \"f64_bytes\": %zu, \"red_f64_random\": %.4g, \"red_f64_walk\": %.4g, "
-           "\"red_f32_random\": %.4g}%s\n",
+           "\"red_f32_random\": %.4g, ",
            c.name, nb, (size_t)nb * 8, n / (ms_r * 1e-3), (nthr * (iters / 64 * 64)) / (ms_w * 1e-3),
-           n / (ms_f * 1e-3), gi < 2 ? "," : "");
+           n / (ms_f * 1e-3));
+    cr.print();
+    printf("}%s\n", gi < 2 ? "," : "");
   }
   printf(" },\n");
   {
@@ -194,7 +248,9 @@ int main() {
     const int it = 4096;
     const float ms = t.best([&] { red_shared<<<blocks, threads, sb * 8>>>(out, it, sb); });
     CK(cudaGetLastError());
-    printf(" \"red_shared_f64_per_s\": %.4g,\n", nthr * it / (ms * 1e-3));
+    printf(" \"red_shared_f64_per_s\": %.4g, ", nthr * it / (ms * 1e-3));
+    clog.print("red_shared_f64_clock");
+    printf(",\n");
     CK(cudaFuncSetAttribute(red_shared_t<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, sb * 8));
     const float msf = t.best([&] { red_shared_t<float><<<blocks, threads, sb * 8>>>(out, it, sb); });
     CK(cudaGetLastError());
@@ -221,8 +277,10 @@ int main() {
     const float ms = t.best([&] { fp64_alu<<<blocks, threads>>>(out, it); });
     CK(cudaGetLastError());
     const double ops = nthr * it * 8 * 2;
-    printf(" \"fp64_alu_ops_per_s\": %.4g,\n \"fp64_lanes_per_sm_at_attr_clock\": %.3g\n}\n", ops / (ms * 1e-3),
+    printf(" \"fp64_alu_ops_per_s\": %.4g,\n \"fp64_lanes_per_sm_at_attr_clock\": %.3g,\n ", ops / (ms * 1e-3),
            ops / (ms * 1e-3) / nsm / (clk * 1e3));
+    clog.print("fp64_alu_clock");
+    printf("\n}\n");
   }
   CK(cudaFree(h));
   CK(cudaFree(out));
