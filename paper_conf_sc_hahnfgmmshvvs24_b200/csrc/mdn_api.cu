@@ -239,7 +239,10 @@ mdn_status run_mdnorm(mdn_grid* g, mdn::MdnParams p, const MatBlock& mb, cudaStr
     g->hit_cap = cap;
     if (cap < want) g->hit_cap_max = cap;  // do not retry the larger size on every call
   }
-  if (!g->d_ctr) MDN_CUDA(cudaMalloc(&g->d_ctr, sizeof(mdn::DevCounters)), "counters");
+  if (!g->d_ctr) {
+    MDN_CUDA(cudaMalloc(&g->d_ctr, sizeof(mdn::DevCounters)), "counters");
+    MDN_CUDA(cudaMemset(g->d_ctr, 0, sizeof(mdn::DevCounters)), "counters");  // the walk keeps them zero
+  }
   p.hit = g->d_hit;
   p.ctr = g->d_ctr;
   // pixels per slab so that every trajectory of the slab can be a hitter, split evenly
@@ -1069,7 +1072,7 @@ mdn_status mdnorm_debug_last_launch(mdn_grid* g, int64_t out[4]) {
     MDN_CUDA(cudaMemcpy(&c, g->d_ctr, sizeof c, cudaMemcpyDeviceToHost), "counters D2H");
   }
   out[0] = g->last_nslab;
-  out[1] = c.nhit;
+  out[1] = c.last_nhit;
   out[2] = mdn::walk_big_claim_threshold(g->g.n[2] > 1, g->num_sms);
   out[3] = g->slab_limit;
   return ok();

@@ -83,7 +83,7 @@ template <typename T>
 __device__ __forceinline__ void priv_flush(const T* h, double* dst, int64_t n) {
   for (int64_t i = threadIdx.x; i < n; i += blockDim.x) {
     const T v = h[i];
-    if (v != T(0)) atomicAdd(dst + i, (double)v);
+    if (v != T(0)) red_add(dst + i, (double)v);
   }
 }
 

@@ -56,9 +56,12 @@ struct SmemEmit {
   }
 };
 
+// red.global.add.f64 stated explicitly (red_add): with a fence anywhere in the kernel (the
+// counters' reset at its end) the compiler otherwise turns atomicAdd into an atomic with a
+// discarded return (ATOMG), and every segment waits for its L2 round trip -- measured 2x slower.
 struct AtomicEmit {
   double* h;
-  __device__ __forceinline__ void operator()(int b, double val) const { atomicAdd(h + b, val); }
+  __device__ __forceinline__ void operator()(int b, double val) const { red_add(h + b, val); }
 };
 
 // Momentum range of a pixel's trajectories: the call's [k_min, k_max], intersected with the
@@ -254,6 +257,10 @@ mdnorm_cull_kernel(const __grid_constant__ MdnParams p, const __grid_constant__ 
     flush_counter(p.stats + 1, c_hit);
     flush_counter(p.stats + 2, c_cross);
   }
+  // launched with programmatic dependent launch: the cull may run while the kernel before it
+  // (e.g. the run's BinMD, which it does not depend on) finishes, but it completes only after that
+  // kernel has, so everything after the walk sees both (no-op without the attribute)
+  asm volatile("griddepcontrol.wait;" ::: "memory");
 }
 
 // ---------------------------------------------------------------- M3-M7: balanced piece walk
@@ -352,10 +359,9 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
       n = __shfl_sync(kFull, n, 0);
       if (b >= nhit) {
         more = false;
-        // this warp claims nothing more: once every warp of every CTA is here (the start of the
-        // end spread) a BinMD launched with programmatic stream serialisation may take the SMs
-        // that walk CTAs leave
-        asm volatile("griddepcontrol.launch_dependents;");
+        // no early launch_dependents here: a cull launched after this walk (the next slab or run
+        // block) reuses the hitter buffer and counters, so it may start only when the walk is
+        // done (the implicit trigger at grid completion)
         break;
       }
       const unsigned nnew = min(n, nhit - b);
@@ -459,6 +465,19 @@ mdnorm_walk_kernel(const __grid_constant__ MdnParams p) {
     priv_flush(sHist, p.norm, p.g.nbins);
   }
   if (kStats) flush_counter(p.stats + 3, c_seg);
+  // the last CTA out returns the counters to zero for the next slab's cull
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    if (atomicAdd(&p.ctr->done, 1u) == gridDim.x - 1) {
+      p.ctr->last_nhit = nhit;
+      p.ctr->nhit = 0;
+      p.ctr->claimed = 0;
+      p.ctr->pclaim = 0;
+      p.ctr->done = 0;
+      __threadfence();
+    }
+  }
 }
 
 // ---------------------------------------------------------------- X2
@@ -608,8 +627,19 @@ cudaError_t launch_cull(const MdnParams& p, const MatBlock& mb, int num_sms, cud
   int per_sm = 0;
   err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kThreads, smem);
   if (err != cudaSuccess) return err;
-  k<<<grid_for(p.plen, num_sms, std::max(per_sm, 1)), kThreads, smem, s>>>(p, mb);
-  return cudaGetLastError();
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)grid_for(p.plen, num_sms, std::max(per_sm, 1)));
+  cfg.blockDim = dim3(kThreads);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  // programmatic dependent launch: cull CTAs take the SMs that the previous kernel's CTAs leave
+  // (a BinMD launched before MDNorm ends unevenly: its in-grid events are clustered)
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, k, p, mb);
 }
 
 
@@ -627,9 +657,7 @@ uint32_t walk_big_claim_threshold(bool d3, int num_sms) {
 
 cudaError_t launch_mdnorm(const MdnParams& p, const MatBlock& mb, int num_sms, cudaStream_t s) {
   if (p.plen == 0 || mb.nmat <= 0) return cudaSuccess;
-  cudaError_t err = cudaMemsetAsync(p.ctr, 0, sizeof(DevCounters), s);
-  if (err != cudaSuccess) return err;
-  err = p.stats ? launch_cull<true>(p, mb, num_sms, s) : launch_cull<false>(p, mb, num_sms, s);
+  cudaError_t err = p.stats ? launch_cull<true>(p, mb, num_sms, s) : launch_cull<false>(p, mb, num_sms, s);
   if (err != cudaSuccess) return err;
   // 2-D slices (a single bin on the last axis, "lBins=1") merge two crossing streams
   const bool d3 = p.g.n[2] > 1;

@@ -55,11 +55,16 @@ struct alignas(16) Hitter {
   int32_t jA, stepG, P;
 };
 
+// Zero at the start of every cull: the walk's last CTA returns them to zero (so no memset sits
+// between a preceding kernel and the cull, which is launched with programmatic dependent launch)
+// and keeps the slab's hitter count in last_nhit (tracing).
 struct DevCounters {
-  unsigned int nhit;     // hitters written by the cull kernel
-  unsigned int claimed;  // hitters claimed by the walk kernel's warps
-  unsigned int pclaim;   // slab pixels claimed by the cull kernel's warps
-  unsigned int pad;
+  unsigned int nhit;      // hitters written by the cull kernel
+  unsigned int claimed;   // hitters claimed by the walk kernel's warps
+  unsigned int pclaim;    // slab pixels claimed by the cull kernel's warps
+  unsigned int done;      // walk CTAs finished
+  unsigned int last_nhit; // hitters of the last slab walked
+  unsigned int pad[3];
 };
 
 struct MdnParams {
