@@ -134,6 +134,26 @@ mdn_status binmd_accumulate_err(mdn_grid *g, const double UB[9], int32_t nops, c
                                 int64_t nevents, const float *events, int64_t stride_floats,
                                 int32_t col_w, int32_t col_e, int32_t col_q, void *stream);
 
+/* MDBox extents ("Mantid's BinMD uses a hierarchy of boxes with equal numbers
+ * of events"; the SaveMD files the workflow reads store them): events (DEVICE,
+ * packed float4 (w, Qx, Qy, Qz), 16-byte aligned) are cut into boxes of box_events consecutive
+ * events (a power of two >= 32; the last box may be shorter) and bounds (DEVICE float[6 * nboxes],
+ * nboxes = ceil(nevents / box_events)) receives each box's (min Qx, min Qy, min Qz, max Qx, max Qy,
+ * max Qz) over its events with finite Q.  One pass over the events, stream-ordered; the extents
+ * belong to the event list and serve every later binmd_accumulate_boxes of it. */
+mdn_status binmd_box_bounds(mdn_grid *g, int64_t nevents, const float *events, int32_t box_events,
+                            float *bounds, void *stream);
+
+/* BinMD of one run's events grouped in MDBoxes with known extents (binmd_box_bounds, or the file's
+ * own): a box whose extent cannot reach the grid under any op (fp64 interval arithmetic on the
+ * extent, widened far beyond rounding) is not read at all; the events of the other boxes take the
+ * binmd_accumulate path.  The result equals binmd_accumulate's on the same events provided every
+ * event's Q lies inside its box's bounds (the caller's contract).  events, bounds: DEVICE
+ * (borrowed until the stream reaches the work); packed float4 layout only. */
+mdn_status binmd_accumulate_boxes(mdn_grid *g, const double UB[9], int32_t nops, const double *ops,
+                                  int64_t nevents, const float *events, int32_t box_events,
+                                  const float *bounds, void *stream);
+
 /* Borrowed device pointers to the fp64 histograms (each nbins_total doubles). */
 mdn_status mdnorm_histograms(mdn_grid *g, void **norm_dev, void **binmd_dev, int64_t *nbins_total);
 

@@ -52,6 +52,8 @@ SIGNATURES = {
     "mdnorm_debug_compose": [P, P, i32, P, i32, P, P, P],
     "mdnorm_debug_set_max_slab": [P, i64],
     "mdnorm_debug_last_launch": [P, P],
+    "binmd_box_bounds": [P, i64, P, i32, P, P],
+    "binmd_accumulate_boxes": [P, P, i32, P, i64, P, i32, P, P],
 }
 _RESTYPES = {"mdn_last_error": C.c_char_p, "mdn_version": C.c_char_p}
 

@@ -56,6 +56,8 @@ struct mdn_grid {
   // runs on plan_stream (it depends on no device data, so it overlaps the MDNorm kernels before
   // it) and the BinMD kernels wait for it
   void* d_btab[2] = {nullptr, nullptr};
+  int32_t* d_blist[2] = {nullptr, nullptr};  // surviving boxes (binmd_accumulate_boxes), count first
+  int64_t blist_cap[2] = {0, 0};
   int btab_i = 0;
   cudaStream_t plan_stream = nullptr;
   cudaEvent_t ev_tab_ready[2] = {nullptr, nullptr};
@@ -357,7 +359,8 @@ mdn_status binmd_host_stream(mdn_grid* g, const MatBlock& mb, int64_t nevents, c
 // B0 of one BinMD call: the plan kernel on plan_stream into the next table buffer, ordered after
 // the last kernels that read that buffer; returns the buffer (the caller's kernels wait on
 // ev_tab_ready and record ev_tab_free after them).
-mdn_status binmd_plan(mdn_grid* g, const MatBlock& mb, const EvLayout& L, cudaStream_t s, int* slot) {
+mdn_status binmd_plan(mdn_grid* g, const MatBlock& mb, const EvLayout& L, cudaStream_t s, int* slot,
+                      const float* box_bounds = nullptr, int64_t nboxes = 0) {
   if (!g->plan_stream) {
     MDN_CUDA(cudaStreamCreateWithFlags(&g->plan_stream, cudaStreamNonBlocking), "plan stream");
     for (int i = 0; i < 2; ++i) {
@@ -368,11 +371,27 @@ mdn_status binmd_plan(mdn_grid* g, const MatBlock& mb, const EvLayout& L, cudaSt
   const int i = g->btab_i ^ 1;
   if (!g->d_btab[i]) MDN_CUDA(cudaMalloc(&g->d_btab[i], mdn::binmd_tables_bytes()), "binmd tables");
 
-  // the plan runs after the caller's work up to its last reset (the start of its accumulation
-  // epoch, as for host-event copies) and after the last kernels that read this buffer
-  if (g->ev_epoch) MDN_CUDA(cudaStreamWaitEvent(g->plan_stream, g->ev_epoch, 0), "wait");
+  // the plan reads only host-side parameters: it waits for nothing but the last kernels that read
+  // this buffer (two calls back), so it runs as soon as the host enqueues it -- typically during
+  // the previous call's kernels -- and is off the critical path
   MDN_CUDA(cudaStreamWaitEvent(g->plan_stream, g->ev_tab_free[i], 0), "wait");
   MDN_CUDA(mdn::launch_binmd_plan(bin_params(g, nullptr, 0, L), mb, g->d_btab[i], g->plan_stream), "binmd plan");
+  if (box_bounds) {  // NEXT #4: the boxes that can reach the grid, after the plan's tables
+    if (g->blist_cap[i] < nboxes + 1) {
+      MDN_CUDA(cudaEventSynchronize(g->ev_tab_free[i]), "sync");
+      cudaFree(g->d_blist[i]);
+      g->d_blist[i] = nullptr;
+      g->blist_cap[i] = 0;
+      MDN_CUDA(cudaMalloc(&g->d_blist[i], sizeof(int32_t) * (size_t)(nboxes + 1)), "box list");
+      g->blist_cap[i] = nboxes + 1;
+    }
+    MDN_CUDA(cudaMemsetAsync(g->d_blist[i], 0, sizeof(int32_t), g->plan_stream), "box count");
+    mdn::BinParams bp = bin_params(g, nullptr, 0, L);
+    bp.tables = g->d_btab[i];
+    MDN_CUDA(mdn::launch_binmd_box_cull(bp, box_bounds, nboxes, g->d_blist[i] + 1,
+                                        reinterpret_cast<unsigned*>(g->d_blist[i]), g->num_sms, g->plan_stream),
+             "box cull");
+  }
   MDN_CUDA(cudaEventRecord(g->ev_tab_ready[i], g->plan_stream), "event record");
   MDN_CUDA(cudaStreamWaitEvent(s, g->ev_tab_ready[i], 0), "wait");
   g->btab_i = i;
@@ -478,6 +497,7 @@ mdn_status mdnorm_destroy(mdn_grid* g) {
   if (g->copy_stream) cudaStreamDestroy(g->copy_stream);
   for (int i = 0; i < 2; ++i) {
     cudaFree(g->d_btab[i]);
+    cudaFree(g->d_blist[i]);
     if (g->ev_tab_ready[i]) cudaEventDestroy(g->ev_tab_ready[i]);
     if (g->ev_tab_free[i]) cudaEventDestroy(g->ev_tab_free[i]);
   }
@@ -783,6 +803,61 @@ mdn_status binmd_accumulate_err(mdn_grid* g, const double UB[9], int32_t nops, c
 mdn_status binmd_accumulate(mdn_grid* g, const double UB[9], int32_t nops, const double* ops, int64_t nevents,
                             const float* events, int64_t stride_floats, int32_t col_w, int32_t col_q, void* stream) {
   return binmd_accumulate_err(g, UB, nops, ops, nevents, events, stride_floats, col_w, -1, col_q, stream);
+}
+
+mdn_status binmd_box_bounds(mdn_grid* g, int64_t nevents, const float* events, int32_t box_events, float* bounds,
+                            void* stream) {
+  if (!g) return fail(MDN_EINVAL, "grid is NULL");
+  if (nevents < 0 || box_events < 32 || (box_events & (box_events - 1)))
+    return fail(MDN_EINVAL, "need nevents >= 0 and box_events a power of two >= 32 (got %lld, %d)",
+                (long long)nevents, box_events);
+  if (nevents == 0) return ok();
+  if (!events || !bounds) return fail(MDN_EINVAL, "events or bounds is NULL");
+  DeviceGuard dg(g->device);
+  if (!is_device_ptr(events) || !is_device_ptr(bounds)) return fail(MDN_EINVAL, "events and bounds must be device arrays");
+  if (reinterpret_cast<uintptr_t>(events) & 15) return fail(MDN_EINVAL, "events must be 16-byte aligned float4 rows");
+  MDN_CUDA(mdn::launch_binmd_box_bounds(reinterpret_cast<const float4*>(events), nevents, box_events, bounds,
+                                        g->num_sms, (cudaStream_t)stream), "box bounds");
+  return ok();
+}
+
+mdn_status binmd_accumulate_boxes(mdn_grid* g, const double UB[9], int32_t nops, const double* ops, int64_t nevents,
+                                  const float* events, int32_t box_events, const float* bounds, void* stream) {
+  if (!g) return fail(MDN_EINVAL, "grid is NULL");
+  mdn_status st;
+  const EvLayout L{4, 0, -1, 1};
+  if ((st = check_matrix(UB, "UB")) != MDN_OK) return st;
+  if ((st = check_ops(nops, ops)) != MDN_OK) return st;
+  if ((st = check_events(nevents, events, L)) != MDN_OK) return st;
+  if (box_events < 32 || (box_events & (box_events - 1)))
+    return fail(MDN_EINVAL, "box_events must be a power of two >= 32 (got %d)", box_events);
+  if (nevents == 0) return ok();
+  if (!bounds) return fail(MDN_EINVAL, "bounds is NULL");
+  DeviceGuard dg(g->device);
+  if (!is_device_ptr(events) || !is_device_ptr(bounds)) return fail(MDN_EINVAL, "events and bounds must be device arrays");
+  if (reinterpret_cast<uintptr_t>(events) & 15) return fail(MDN_EINVAL, "events must be 16-byte aligned float4 rows");
+  cudaStream_t s = (cudaStream_t)stream;
+  MatBlock mb{};
+  mb.compose = 1;
+  mb.nops = nops;
+  mb.nmat = nops;
+  std::memcpy(mb.UB, UB, sizeof mb.UB);
+  std::memcpy(mb.W, g->W, sizeof mb.W);
+  std::memcpy(mb.u.c.ops, ops, sizeof(double) * 9 * nops);
+  const int64_t nboxes = (nevents + box_events - 1) / box_events;
+  int slot = 0;
+  if ((st = binmd_plan(g, mb, L, s, &slot, bounds, nboxes)) != MDN_OK) return st;
+  mdn::BinParams p = bin_params(g, events, nevents, L);
+  p.tables = g->d_btab[slot];
+  p.box_list = g->d_blist[slot] + 1;
+  p.box_count = reinterpret_cast<const unsigned*>(g->d_blist[slot]);
+  int lg = 0;
+  while ((32 << lg) < box_events) ++lg;
+  p.box_log2 = lg;
+  MDN_CUDA(mdn::launch_binmd(p, mb, g->num_sms, s), "binmd kernel");
+  g->path[1] = mdn::last_binmd_path();
+  MDN_CUDA(cudaEventRecord(g->ev_tab_free[slot], s), "event record");
+  return ok();
 }
 
 mdn_status mdnorm_histograms(mdn_grid* g, void** norm_dev, void** binmd_dev, int64_t* nbins_total) {

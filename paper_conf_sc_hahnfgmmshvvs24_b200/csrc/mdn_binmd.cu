@@ -342,7 +342,7 @@ __device__ __forceinline__ float4 load_event(const BinParams& p, int64_t e) {
 
 // The event loop for kNC register classes: grid-stride over warp-contiguous 32-event blocks,
 // two blocks prefetched ahead (three float4 per lane in flight: the event stream is the roof).
-template <int kNC, bool kPacked, bool kStats, int kPriv>
+template <int kNC, bool kPacked, bool kStats, int kPriv, bool kBoxes>
 __device__ __forceinline__ void binmd_loop(const BinParams& p, const MatBlock& mb, const BinTables& T,
                                            float4* qv, unsigned* qk, float* qe, priv_t<kPriv>* hb,
                                            priv_t<kPriv>* he, unsigned long long& c_pairs,
@@ -372,15 +372,27 @@ __device__ __forceinline__ void binmd_loop(const BinParams& p, const MatBlock& m
   // Q-ordered stream (a Bragg peak, the slab) are spread over all SMs (measured: per-SM active
   // cycles max / mean 1.38 with CTA-contiguous blocks on the CORELLI slab).
   const int64_t base0 = ((int64_t)(threadIdx.x >> 5) * gridDim.x + blockIdx.x) * 32;  // warp-uniform
-  // rounds of this warp, and of this lane (they differ only in the last, ragged block)
   const int64_t n = p.nevents;
-  const int rounds = base0 < n ? (int)((n - 1 - base0) / stride) + 1 : 0;
+  // MDBox mode: the same interleave over the 32-event blocks of the listed boxes only
+  const int64_t nvb = kBoxes ? ((int64_t)*p.box_count << p.box_log2) * 32 : n;
+  // rounds of this warp, and of this lane (they differ only in the last, ragged block)
+  const int rounds = base0 < nvb ? (int)((nvb - 1 - base0) / stride) + 1 : 0;
   const int lrounds = base0 + lane < n ? (int)((n - 1 - base0 - lane) / stride) + 1 : 0;
   // event of this lane in round r: e0 + r stride (64-bit only in the address arithmetic)
   const int64_t e0 = base0 + lane;
-  auto ld = [&](int r, float& e2) {
-    if (r < lrounds) {
-      const int64_t e = e0 + (int64_t)r * stride;
+  auto ld = [&](int r, float& e2, bool& valid) {
+    int64_t e;
+    if constexpr (kBoxes) {
+      const int64_t vb = (base0 >> 5) + (int64_t)r * (stride >> 5);  // virtual block of round r
+      const int64_t bpb_mask = ((int64_t)1 << p.box_log2) - 1;
+      e = r < rounds ? (((int64_t)__ldg(p.box_list + (vb >> p.box_log2)) << p.box_log2) + (vb & bpb_mask)) * 32 + lane
+                     : n;
+      valid = e < n;
+    } else {
+      e = e0 + (int64_t)r * stride;
+      valid = r < lrounds;
+    }
+    if (valid) {
       if (has_err) e2 = __ldcs(p.events + e * p.stride + p.col_e);
       return load_event<kPacked>(p, e);
     }
@@ -407,14 +419,15 @@ __device__ __forceinline__ void binmd_loop(const BinParams& p, const MatBlock& m
   // whose load is in flight would wait for that load).
   float4 ev[kDepth];
   float ex[kDepth] = {};
+  bool vd[kDepth];
 #pragma unroll
-  for (int u = 0; u < kDepth; ++u) ev[u] = ld(u, ex[u]);
+  for (int u = 0; u < kDepth; ++u) ev[u] = ld(u, ex[u], vd[u]);
   for (int r = 0;;) {
 #pragma unroll
     for (int u = 0; u < kDepth; ++u) {
       if (r >= rounds) goto done;
-      test(ev[u], ex[u], r < lrounds);
-      ev[u] = ld(r + kDepth, ex[u]);
+      test(ev[u], ex[u], vd[u]);
+      ev[u] = ld(r + kDepth, ex[u], vd[u]);
       ++r;
     }
     // one drain site per kDepth blocks (the ring holds kDepth x 32 + 31 entries): the member code
@@ -447,7 +460,7 @@ __device__ __forceinline__ void load_tables(const void* g, BinTables& T) {
 // One thread per event (grid-stride).  kPriv: 0 = global fp64 red.add, 1 / 2 = a private fp64 /
 // fp32 histogram per CTA in shared memory (binmd, then err2 when the error column is read),
 // flushed into the global one at the end.
-template <bool kPacked, bool kStats, int kPriv>
+template <bool kPacked, bool kStats, int kPriv, bool kBoxes = false>
 __global__ void __launch_bounds__(bin_threads(kPriv), kPriv ? 2 : kBinMinBlocks)
 binmd_kernel(const __grid_constant__ BinParams p, const __grid_constant__ MatBlock mb) {
   constexpr int kBT = bin_threads(kPriv);
@@ -477,11 +490,11 @@ binmd_kernel(const __grid_constant__ BinParams p, const __grid_constant__ MatBlo
   unsigned long long c_pairs = 0, c_in = 0;
   const int ncls = T.ncls;
   if (ncls <= 1)
-    binmd_loop<1, kPacked, kStats, kPriv>(p, mb, T, qv, qk, qe, hb, he, c_pairs, c_in);
+    binmd_loop<1, kPacked, kStats, kPriv, kBoxes>(p, mb, T, qv, qk, qe, hb, he, c_pairs, c_in);
   else if (ncls <= 2)
-    binmd_loop<2, kPacked, kStats, kPriv>(p, mb, T, qv, qk, qe, hb, he, c_pairs, c_in);
+    binmd_loop<2, kPacked, kStats, kPriv, kBoxes>(p, mb, T, qv, qk, qe, hb, he, c_pairs, c_in);
   else
-    binmd_loop<0, kPacked, kStats, kPriv>(p, mb, T, qv, qk, qe, hb, he, c_pairs, c_in);
+    binmd_loop<0, kPacked, kStats, kPriv, kBoxes>(p, mb, T, qv, qk, qe, hb, he, c_pairs, c_in);
   if (kPriv) {
     __syncthreads();
     priv_flush(hb, p.binmd, p.g.nbins);
@@ -520,10 +533,96 @@ debug_bins_kernel(const __grid_constant__ BinParams p, const __grid_constant__ M
   }
 }
 
-template <bool kPacked, bool kStats, int kPriv>
+// ---------------------------------------------------------------- NEXT #4: MDBox extents
+// Q extents of boxes of box_events consecutive packed events (the last box may be shorter): one
+// warp per box, coalesced float4 loads, warp min / max.  bounds[6 b ..] = (min q0, q1, q2, max q0,
+// q1, q2).
+__global__ void __launch_bounds__(kThreads) binmd_box_bounds_kernel(const float4* __restrict__ ev, int64_t n,
+                                                                    int32_t box_events, float* __restrict__ bounds,
+                                                                    int64_t nboxes) {
+  const int lane = threadIdx.x & 31;
+  const int64_t nw = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t b = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); b < nboxes; b += nw) {
+    float lo0 = CUDART_INF_F, lo1 = CUDART_INF_F, lo2 = CUDART_INF_F;
+    float hi0 = -CUDART_INF_F, hi1 = -CUDART_INF_F, hi2 = -CUDART_INF_F;
+    const int64_t e1 = min(n, (b + 1) * (int64_t)box_events);
+    for (int64_t e = b * (int64_t)box_events + lane; e < e1; e += 32) {
+      const float4 v = __ldcs(ev + e);
+      lo0 = fminf(lo0, v.y); lo1 = fminf(lo1, v.z); lo2 = fminf(lo2, v.w);
+      hi0 = fmaxf(hi0, v.y); hi1 = fmaxf(hi1, v.z); hi2 = fmaxf(hi2, v.w);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      lo0 = fminf(lo0, __shfl_xor_sync(kFull, lo0, o)); lo1 = fminf(lo1, __shfl_xor_sync(kFull, lo1, o));
+      lo2 = fminf(lo2, __shfl_xor_sync(kFull, lo2, o)); hi0 = fmaxf(hi0, __shfl_xor_sync(kFull, hi0, o));
+      hi1 = fmaxf(hi1, __shfl_xor_sync(kFull, hi1, o)); hi2 = fmaxf(hi2, __shfl_xor_sync(kFull, hi2, o));
+    }
+    if (lane < 6) bounds[6 * b + lane] = lane == 0 ? lo0 : lane == 1 ? lo1 : lane == 2 ? lo2 : lane == 3 ? hi0 : lane == 4 ? hi1 : hi2;
+  }
+}
+
+// The boxes whose extent can reach the grid under some matrix of the launch (thread per box):
+// x_a = N_a . q over the box is enclosed by [sum_i min(N_ai lo_i, N_ai hi_i), sum_i max(..)] in
+// fp64; the box is dropped only when, for every matrix, some axis has t = (x - lo) s entirely
+// below -eps or at or above n + eps (eps = 1e-6 (n + |lo s| + 1): far beyond the rounding of the
+// fp64 enclosure and of the definition's own t).  Survivors are appended in any order.
+__global__ void __launch_bounds__(kThreads) binmd_box_cull_kernel(const __grid_constant__ BinParams p,
+                                                                  const float* __restrict__ bounds, int64_t nboxes,
+                                                                  int32_t* __restrict__ list,
+                                                                  unsigned* __restrict__ count) {
+  __shared__ double sN[kMaxMats * 9];
+  __shared__ int snmat;
+  const BinTables* gt = static_cast<const BinTables*>(p.tables);
+  if (threadIdx.x == 0) snmat = gt->sCls[gt->ncls];  // number of matrices (sCls[ncls] = nmat)
+  __syncthreads();
+  const int nmat = snmat;
+  for (int i = threadIdx.x; i < 9 * nmat; i += blockDim.x) sN[i] = gt->sN[i];
+  __syncthreads();
+  const int lane = threadIdx.x & 31;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t b0 = (int64_t)blockIdx.x * blockDim.x; b0 < nboxes; b0 += stride) {
+    const int64_t b = b0 + threadIdx.x;
+    bool keep = false;
+    if (b < nboxes) {
+      double lo[3], hi[3];
+      for (int i = 0; i < 3; ++i) {
+        lo[i] = (double)bounds[6 * b + i];
+        hi[i] = (double)bounds[6 * b + 3 + i];
+      }
+      // no finite-Q event (fminf / fmaxf skip NaN): every event of the box is outside by definition
+      const bool empty = !(lo[0] <= hi[0]);
+      if (!empty) {
+        for (int m = 0; m < nmat && !keep; ++m) {
+          bool miss = false;
+          for (int a = 0; a < 3 && !miss; ++a) {
+            const double* r = sN + 9 * m + 3 * a;
+            double xl = 0.0, xh = 0.0;
+            for (int i = 0; i < 3; ++i) {
+              const double u = r[i] * lo[i], v = r[i] * hi[i];
+              xl += fmin(u, v);
+              xh += fmax(u, v);
+            }
+            const double s = p.g.s[a], l = p.g.lo[a], nb = p.g.nd[a];
+            const double eps = 1e-6 * (nb + fabs(l * s) + 1.0);
+            const double tl = (xl - l) * s, th = (xh - l) * s;
+            miss = th < -eps || tl >= nb + eps;  // NaN compares false: kept
+          }
+          keep = !miss;
+        }
+      }
+    }
+    const unsigned bal = __ballot_sync(kFull, keep);
+    unsigned at = 0;
+    if (lane == 0 && bal) at = atomicAdd(count, (unsigned)__popc(bal));
+    at = __shfl_sync(kFull, at, 0);
+    if (keep) list[at + __popc(bal & ((1u << lane) - 1u))] = (int32_t)b;
+  }
+}
+
+template <bool kPacked, bool kStats, int kPriv, bool kBoxes = false>
 cudaError_t launch_binmd_t(const BinParams& p, const MatBlock& mb, int num_sms, size_t smem, cudaStream_t s) {
   constexpr int threads = bin_threads(kPriv);
-  auto k = binmd_kernel<kPacked, kStats, kPriv>;
+  auto k = binmd_kernel<kPacked, kStats, kPriv, kBoxes>;
   smem += queue_bytes(threads);
   cudaError_t err = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (err != cudaSuccess) return err;
@@ -537,6 +636,9 @@ cudaError_t launch_binmd_t(const BinParams& p, const MatBlock& mb, int num_sms, 
 template <int kPriv>
 cudaError_t launch_binmd_p(const BinParams& p, const MatBlock& mb, bool packed, int num_sms, size_t smem,
                            cudaStream_t s) {
+  if (p.box_list)  // MDBox mode: packed float4 events only (checked by the API)
+    return p.stats ? launch_binmd_t<true, true, kPriv, true>(p, mb, num_sms, smem, s)
+                   : launch_binmd_t<true, false, kPriv, true>(p, mb, num_sms, smem, s);
   if (packed) return p.stats ? launch_binmd_t<true, true, kPriv>(p, mb, num_sms, smem, s)
                              : launch_binmd_t<true, false, kPriv>(p, mb, num_sms, smem, s);
   return p.stats ? launch_binmd_t<false, true, kPriv>(p, mb, num_sms, smem, s)
@@ -589,6 +691,22 @@ int last_binmd_path() { return g_last_binmd_path; }
 
 
 size_t binmd_tables_bytes() { return sizeof(BinTables); }
+
+cudaError_t launch_binmd_box_bounds(const float4* events, int64_t nevents, int32_t box_events, float* bounds,
+                                    int num_sms, cudaStream_t s) {
+  const int64_t nboxes = (nevents + box_events - 1) / box_events;
+  if (nboxes <= 0) return cudaSuccess;
+  binmd_box_bounds_kernel<<<grid_for(nboxes * 32, num_sms, 8), kThreads, 0, s>>>(events, nevents, box_events,
+                                                                                 bounds, nboxes);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_binmd_box_cull(const BinParams& p, const float* bounds, int64_t nboxes, int32_t* list,
+                                  unsigned* count, int num_sms, cudaStream_t s) {
+  if (nboxes <= 0) return cudaSuccess;
+  binmd_box_cull_kernel<<<grid_for(nboxes, num_sms, 4), kThreads, 0, s>>>(p, bounds, nboxes, list, count);
+  return cudaGetLastError();
+}
 
 cudaError_t launch_binmd_plan(const BinParams& p, const MatBlock& mb, void* tables, cudaStream_t s) {
   binmd_plan_kernel<<<1, kThreads, 0, s>>>(p, mb, static_cast<BinTables*>(tables));

@@ -101,6 +101,11 @@ struct BinParams {
   double* err2;            // fp64 error-squared histogram (nbins), used when col_e >= 0
   unsigned long long* stats;  // nullptr, or [.., .., .., .., pairs, inside] (+= per launch)
   const void* tables;      // the launch's BinTables in global memory (launch_binmd_plan)
+  // MDBox mode (NEXT #4, binmd_accumulate_boxes): only the boxes listed in box_list (box_count of
+  // them, written by launch_binmd_box_cull) are read; box b = events [b box_events, (b+1) box_events)
+  const int32_t* box_list;
+  const unsigned* box_count;
+  int32_t box_log2;        // log2(box_events / 32)
 };
 
 // launchers (return the launch's cudaError_t)
@@ -116,6 +121,13 @@ cudaError_t launch_binmd(const BinParams& p, const MatBlock& mb, int num_sms, cu
 // of binmd_tables_bytes()), one CTA; binmd_kernel reads them (BinParams::tables).
 size_t binmd_tables_bytes();
 cudaError_t launch_binmd_plan(const BinParams& p, const MatBlock& mb, void* tables, cudaStream_t s);
+// NEXT #4: Q extents of boxes of box_events consecutive packed events (one pass), and the list of
+// boxes that can reach the grid under some op of the launch's tables (conservative fp64 interval
+// arithmetic); count must be zero before the cull.
+cudaError_t launch_binmd_box_bounds(const float4* events, int64_t nevents, int32_t box_events, float* bounds,
+                                    int num_sms, cudaStream_t s);
+cudaError_t launch_binmd_box_cull(const BinParams& p, const float* bounds, int64_t nboxes, int32_t* list,
+                                  unsigned* count, int num_sms, cudaStream_t s);
 // Accumulation path chosen for the last launch_mdnorm / launch_binmd on this thread (tracing and
 // tests): 0 = global fp64 red.add, 1 = shared-memory fp64 partials, 2 = shared-memory fp32 partials.
 int last_mdnorm_path();

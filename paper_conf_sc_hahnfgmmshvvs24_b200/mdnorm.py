@@ -375,3 +375,28 @@ def mdnorm_debug_last_launch(g: Grid) -> dict:
     out = np.zeros(4, np.int64)
     check(load().mdnorm_debug_last_launch(g.handle, out.ctypes.data), "mdnorm_debug_last_launch")
     return dict(zip(("slabs", "hitters", "big_claim_threshold", "slab_limit"), (int(x) for x in out)))
+
+
+def binmd_box_bounds(g: Grid, events, box_events=1024, bounds=None, stream=None):
+    """MDBox extents (NEXT #4) of packed float4 CUDA events: a CUDA float32 tensor [nboxes, 6]
+    (allocated if None) of (min Qx, Qy, Qz, max Qx, Qy, Qz) per box of box_events events."""
+    import torch
+    if not (_is_torch(events) and events.is_cuda and events.dtype == torch.float32 and events.is_contiguous()):
+        raise ValueError("events must be a contiguous float32 CUDA tensor [n, 4]")
+    n = events.numel() // 4
+    nboxes = -(-n // int(box_events))
+    if bounds is None:
+        bounds = torch.empty((nboxes, 6), dtype=torch.float32, device=events.device)
+    check(load().binmd_box_bounds(g.handle, n, events.data_ptr(), int(box_events), bounds.data_ptr(),
+                                  _stream(stream, g.device)), "binmd_box_bounds")
+    return bounds
+
+
+def binmd_accumulate_boxes(g: Grid, UB, ops, events, box_events, bounds, stream=None) -> None:
+    """BinMD over MDBoxes with known extents: boxes that cannot reach the grid are not read."""
+    ops = np.ascontiguousarray(ops, dtype=np.float64).reshape(-1, 9)
+    n = events.numel() // 4
+    UB_p, UB_k = _arg(UB, np.float64, 9)
+    check(load().binmd_accumulate_boxes(g.handle, UB_p, len(ops), ops.ctypes.data, n, events.data_ptr(),
+                                        int(box_events), bounds.data_ptr(), _stream(stream, g.device)),
+          "binmd_accumulate_boxes")

@@ -20,7 +20,7 @@ import subprocess
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 PROF = os.path.join(ROOT, "profiles")
-OURS = re.compile(r"(mdnorm_cull_kernel|mdnorm_walk_kernel|binmd_kernel|xs_kernel|debug_\w+|pixels_prepare_kernel)")
+OURS = re.compile(r"(mdnorm_cull_kernel|mdnorm_walk_kernel|binmd_plan_kernel|binmd_kernel|xs_kernel|debug_\w+|pixels_prepare_kernel)")
 
 KEY_METRICS = [
     "gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",
@@ -31,6 +31,15 @@ KEY_METRICS = [
     "lts__t_sectors_srcunit_tex_op_red.sum", "lts__t_sectors_srcunit_tex_op_red.sum.pct_of_peak_sustained_elapsed",
     "lts__t_sectors.sum.pct_of_peak_sustained_elapsed", "launch__registers_per_thread", "launch__grid_size",
     "launch__block_size", "smsp__issue_active.avg.pct_of_peak_sustained_active",
+    # the L1TEX data pipe (shared-memory look-ups and global reductions share it: the walk's
+    # binding resource), its shared-memory part, bank conflicts, global-reduction wavefronts
+    "l1tex__data_pipe_lsu_wavefronts.sum.pct_of_peak_sustained_elapsed",
+    "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum",
+    "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum.pct_of_peak_sustained_elapsed",
+    "l1tex__data_bank_conflicts_pipe_lsu_mem_shared.sum",
+    "l1tex__t_output_wavefronts_pipe_lsu_mem_global_op_red.sum.pct_of_peak_sustained_elapsed",
+    "smsp__average_warps_issue_stalled_long_scoreboard_per_issue_active.ratio",
+    "sm__cycles_active.avg", "sm__cycles_active.max", "dram__throughput.avg.pct_of_peak_sustained_elapsed",
 ]
 
 
@@ -115,14 +124,16 @@ def full(path, tag):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--tag", required=True)
-    ap.add_argument("--launches", default=os.path.join(ROOT, "gpurun_out", "launches.csv"))
-    ap.add_argument("--full", default=os.path.join(ROOT, "gpurun_out", "prof_full.ncu-rep"))
+    ap.add_argument("--launches", default=None)
+    ap.add_argument("--full", default=None)
     a = ap.parse_args()
     os.makedirs(PROF, exist_ok=True)
-    if os.path.exists(a.launches):
-        launches(a.launches, a.tag)
-    if os.path.exists(a.full):
-        full(a.full, a.tag)
+    lp = a.launches or os.path.join(ROOT, "gpurun_out", f"{a.tag}_launches.csv")
+    fp = a.full or os.path.join(ROOT, "gpurun_out", f"{a.tag}_full.ncu-rep")
+    if os.path.exists(lp):
+        launches(lp, a.tag)
+    if os.path.exists(fp):
+        full(fp, a.tag)
 
 
 if __name__ == "__main__":

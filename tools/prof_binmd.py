@@ -21,6 +21,7 @@ def main():
     ap.add_argument("--order", default="morton")
     ap.add_argument("--ncu", action="store_true", help="3 launches only (for ncu -k binmd_kernel)")
     ap.add_argument("--sizes", default="1024,151552,1000000,3000000,10000000")
+    ap.add_argument("--boxes", type=int, default=0, help="also time binmd_accumulate_boxes with this box size")
     args = ap.parse_args()
     import numpy as np
     import torch
@@ -53,6 +54,26 @@ def main():
         out[n] = (float(np.median(ts)), float(np.min(ts)))
         print(json.dumps({"lib": os.path.basename(os.environ.get("MDN_LIB_PATH", "default")), "events": n, "median_ms": out[n][0], "min_ms": out[n][1],
                           "GB/s": 16 * n / out[n][0] / 1e6}), flush=True)
+        if args.boxes:
+            res = {}
+            bounds = m.binmd_box_bounds(g, sub, args.boxes)
+            for what in ("bounds", "boxes"):
+                ts = []
+                for it in range(args.iters + 3):
+                    flush.zero_()
+                    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    a.record()
+                    if what == "bounds":
+                        m.binmd_box_bounds(g, sub, args.boxes, bounds)
+                    else:
+                        m.binmd_accumulate_boxes(g, wl.UB, wl.ops, sub, args.boxes, bounds)
+                    b.record()
+                    torch.cuda.synchronize()
+                    if it >= 3:
+                        ts.append(a.elapsed_time(b))
+                res[what] = float(np.median(ts))
+            print(json.dumps({"events": n, "box_events": args.boxes, "bounds_ms": res["bounds"],
+                              "binmd_boxes_ms": res["boxes"]}), flush=True)
 
 
 if __name__ == "__main__":
