@@ -56,6 +56,16 @@ def measured_peaks():
     return {"hbm_gbs": 6650.0, "sm_max_mhz": 1965.0}, "fallback"
 
 
+def ncu_binding():
+    """Per-kernel utilisation of the resources that can bind it (tools/ncu_summarize.py from the
+    committed ncu --set full capture)."""
+    p = os.path.join(ROOT, "profiles", "ncu_binding.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            return json.load(f)
+    return {"kernels": {}}
+
+
 def ncu_traffic():
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(p):
@@ -575,10 +585,27 @@ def run_ours(args, rank, world, local_rank):
         xs_bytes = 24 * g.nbins_total
         kernels["xs_kernel"] = {"bound": "hbm", "achieved": xs_bytes / tx / 1e9, "peak": hbm, "unit": "GB/s",
                                 "frac": xs_bytes / tx / 1e9 / hbm, "ms": ph_ms["xs"]}
+    nb = ncu_binding()
+    walk = nb["kernels"].get("mdnorm_walk_kernel", {})
+    if walk:
+        kernels["mdnorm"]["binding"] = {
+            "resource": "L1TEX data pipe: shared-memory flux look-ups + global fp64 reductions (walk)",
+            "ncu_walk": walk, "ncu_cull": nb["kernels"].get("mdnorm_cull_kernel", {}), "source": nb.get("source")}
+    if nb["kernels"].get("binmd_kernel"):
+        kernels["binmd_kernel"]["binding"] = {
+            "resource": "latency and per-SM imbalance of the in-grid (event, op) decisions and their reductions",
+            "ncu": nb["kernels"]["binmd_kernel"], "source": nb.get("source")}
     dom = max(("mdnorm", "binmd_kernel"), key=lambda k: kernels[k]["ms"])
     roof = {k: kernels[dom][k] for k in ("bound", "achieved", "peak", "unit", "frac", "traffic")}
     roof["kernel"] = kernels[dom].get("kernels", dom)
     roof["peak_source"] = kernels[dom].get("peak_source", f"{peaks_src}: MEASURED_PEAKS.json hbm_gbs")
+    if "binding" in kernels[dom]:
+        b = kernels[dom]["binding"]
+        w = b.get("ncu_walk", b.get("ncu", {}))
+        roof["binding_resource"] = {"resource": b["resource"],
+                                    "l1tex_data_pipe_pct_of_peak": w.get("l1tex_data_pipe_pct"),
+                                    "l2_red_sectors_pct_of_peak": w.get("l2_red_sectors_pct"),
+                                    "source": b.get("source")}
 
     # our kernels per step: cull + walk per slab of every launch block (16 runs per block), one
     # binmd per run, the divide on rank 0

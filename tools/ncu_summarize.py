@@ -116,6 +116,28 @@ def full(path, tag):
             pass
     with open(os.path.join(PROF, f"{tag}_ncu_full.md"), "w") as f:
         f.write("\n".join(lines) + "\n")
+    # per kernel: the utilisation of the resources that can bind it (bench.py quotes them beside
+    # the roofline fraction)
+    binding = {}
+    pick = {"l1tex_data_pipe_pct": "l1tex__data_pipe_lsu_wavefronts.sum.pct_of_peak_sustained_elapsed",
+            "shared_wavefronts_pct": "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum.pct_of_peak_sustained_elapsed",
+            "l2_red_sectors_pct": "lts__t_sectors_srcunit_tex_op_red.sum.pct_of_peak_sustained_elapsed",
+            "issue_active_pct": "smsp__issue_active.avg.pct_of_peak_sustained_active",
+            "fp64_pipe_pct": "sm__pipe_fp64_cycles_active.avg.pct_of_peak_sustained_active",
+            "dram_pct": "dram__throughput.avg.pct_of_peak_sustained_elapsed",
+            "sm_cycles_active_avg": "sm__cycles_active.avg", "sm_cycles_active_max": "sm__cycles_active.max"}
+    for k, rs in per.items():
+        r = rs[0]
+        d = {}
+        for name, m in pick.items():
+            if m in h:
+                try:
+                    d[name] = float(r[h.index(m)].replace(",", ""))
+                except ValueError:
+                    pass
+        binding[k.split("<")[0]] = d
+    with open(os.path.join(PROF, "ncu_binding.json"), "w") as f:
+        json.dump({"source": f"profiles/{tag}_ncu_full.md", "kernels": binding}, f, indent=1)
     with open(traffic_p, "w") as f:
         json.dump(traffic, f, indent=1)
     print("\n".join(lines[:60]))
