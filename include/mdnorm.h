@@ -255,6 +255,13 @@ mdn_status mdnorm_debug_set_max_slab(mdn_grid *g, int64_t max_traj);
  * Synchronises the device. */
 mdn_status mdnorm_debug_last_launch(mdn_grid *g, int64_t out[4]);
 
+/* The interval guess mdnorm_set_flux[_tables] chose for flux table `table` (HOST double[2]):
+ * {mode: 0 none, 1 knots near-uniform in k, 2 near-uniform in 1/k (wavelength); the fraction of
+ * the table's k range on which the fp32 guess names the interval (0 for mode 0)}.  The guess only
+ * proposes an interval that the exact comparisons kappa_i <= x < kappa_{i+1} then accept or
+ * reject, so it never changes a value.  MDN_EINVAL: NULL argument or no such table. */
+mdn_status mdnorm_debug_flux_guess(mdn_grid *g, int32_t table, double out[2]);
+
 /* M_{r,s} / N_s exactly as the kernels compose them (device code; HOST outputs).  M: double
  * [nruns*nops][9] run-major; N: double[nops][9].  Synchronous (test entry point). */
 mdn_status mdnorm_debug_compose(mdn_grid *g, const double UB[9], int32_t nruns, const double *R,

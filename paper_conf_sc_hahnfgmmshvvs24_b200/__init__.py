@@ -12,6 +12,6 @@ from .mdnorm import (  # noqa: F401
     mdnorm_set_pixel_krange, mdnorm_set_flux_tables, binmd_accumulate_err, mdnorm_error_histogram, mdnorm_cross_section_err,
     mdnorm_accumulate_matrices, binmd_accumulate_matrices, mdnorm_debug_trajectories,
     binmd_debug_bins, mdnorm_debug_compose, packed_histograms, mdn_divide,
-    mdnorm_debug_set_max_slab, mdnorm_debug_last_launch, binmd_box_bounds, binmd_accumulate_boxes,
+    mdnorm_debug_set_max_slab, mdnorm_debug_last_launch, mdnorm_debug_flux_guess, binmd_box_bounds, binmd_accumulate_boxes,
 )
 from .dist import plan_shards, reduce_packed, reduce_scatter_packed, RankPlan  # noqa: F401

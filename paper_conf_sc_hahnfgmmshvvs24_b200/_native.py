@@ -52,6 +52,7 @@ SIGNATURES = {
     "mdnorm_debug_compose": [P, P, i32, P, i32, P, P, P],
     "mdnorm_debug_set_max_slab": [P, i64],
     "mdnorm_debug_last_launch": [P, P],
+    "mdnorm_debug_flux_guess": [P, i32, P],
     "binmd_box_bounds": [P, i64, P, i32, P, P],
     "binmd_accumulate_boxes": [P, P, i32, P, i64, P, i32, P, P],
 }
@@ -82,7 +83,10 @@ def load() -> C.CDLL:
                 f"{LIB_PATH} is missing: build it with `python -m paper_conf_sc_hahnfgmmshvvs24_b200.build` "
                 "(there is no CPU fallback)")
         lib = C.CDLL(LIB_PATH)
+        dev_variant = "MDN_LIB_PATH" in os.environ  # tools/ A/B builds may predate newer debug entries
         for name, args in SIGNATURES.items():
+            if dev_variant and not hasattr(lib, name):
+                continue
             fn = getattr(lib, name)
             fn.argtypes = args
             fn.restype = _RESTYPES.get(name, C.c_int)

@@ -35,6 +35,7 @@ struct mdn_grid {
   int32_t* d_ptab = nullptr;  // pixel -> flux table (several tables only)
   int32_t nftables = 0;
   mdn::FluxView flux0{};      // view of table 0 (device pointers)
+  std::vector<double> fguess_hit;  // per flux table: fraction of the k range the interval guess names
   mdn::Hitter* d_hit = nullptr;       // cull -> walk hand-off buffer
   uint32_t hit_cap = 0;
   uint32_t hit_cap_max = 0;  // kMaxSlab, lowered if the device cannot hold that buffer
@@ -572,7 +573,45 @@ struct HostFluxTable {
   std::vector<int> tab;
   double k_first, F_first, k_last, F_last, inv_cell;
   int n, ntab;
+  float ga = 0.f, gb = 0.f;
+  int gmode = 0;
+  double ghit = 0.0;
 };
+
+// Interval guess for flux_guess (mdn_device.cuh): fit i ~ (T(x) - T(kappa_0)) / dT for T(x) = x
+// and T(x) = 1/x (knots uniform in wavelength), measure on 64 points per interval spread evenly
+// over [kappa_0, kappa_{n-1}] how often the fp32 guess names x's interval, and keep the better
+// transform if it is right at least kFluxGuessMin of the time (the guess never decides a value:
+// a wrong one falls back to the cell-table search).
+constexpr double kFluxGuessMin = 0.9;
+void fit_flux_guess(const double* hk, int64_t n, HostFluxTable& t) {
+  if (n > (1 << 24)) return;
+  double best = 0.0;
+  for (int mode = 1; mode <= 2; ++mode) {
+    const double T0 = mode == 1 ? hk[0] : 1.0 / hk[0], T1 = mode == 1 ? hk[n - 1] : 1.0 / hk[n - 1];
+    const double dT = (T1 - T0) / (double)(n - 1);
+    if (!std::isfinite(dT) || dT == 0.0) continue;
+    const float ga = (float)(1.0 / dT), gb = (float)(-T0 / dT);
+    const int64_t npts = std::min<int64_t>(64 * (n - 1), 1 << 22);
+    int64_t hit = 0, j = 0;
+    for (int64_t s = 0; s < npts; ++s) {
+      const double x = hk[0] + (hk[n - 1] - hk[0]) * ((double)s + 0.5) / (double)npts;
+      while (j + 2 < n && hk[j + 1] <= x) ++j;  // x's interval
+      const float xf = (float)x;
+      const float u = mode == 1 ? xf : 1.0f / xf;
+      const int64_t g = std::min<int64_t>(std::max<int64_t>((int64_t)std::floor(std::fma(u, ga, gb)), 0), n - 2);
+      hit += g == j;
+    }
+    const double frac = (double)hit / (double)npts;
+    if (frac >= kFluxGuessMin && frac > best) {
+      best = frac;
+      t.ghit = frac;
+      t.gmode = mode;
+      t.ga = ga;
+      t.gb = gb;
+    }
+  }
+}
 
 mdn_status build_flux_table(const double* hk, const double* hF, int64_t n, HostFluxTable& t) {
   if (n < 2 || n > (1 << 28)) return fail(MDN_EINVAL, "a flux table needs 2 .. 2^28 knots (got %lld)", (long long)n);
@@ -620,6 +659,7 @@ mdn_status build_flux_table(const double* hk, const double* hF, int64_t n, HostF
   t.F_last = hF[n - 1];
   t.n = (int)n;
   t.ntab = ntab;
+  fit_flux_guess(hk, n, t);
   return MDN_OK;
 }
 
@@ -703,6 +743,9 @@ mdn_status mdnorm_set_flux_tables(mdn_grid* g, int32_t ntables, const int64_t* o
     v.inv_cell = tabs[t].inv_cell;
     v.n = tabs[t].n;
     v.ntab = tabs[t].ntab;
+    v.ga = tabs[t].ga;
+    v.gb = tabs[t].gb;
+    v.gmode = tabs[t].gmode;
   }
   if (e == cudaSuccess) e = cudaMemcpy(d, all.data(), sizeof(double) * all.size(), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(tab, all_tab.data(), sizeof(int) * ntb, cudaMemcpyHostToDevice);
@@ -725,6 +768,8 @@ mdn_status mdnorm_set_flux_tables(mdn_grid* g, int32_t ntables, const int64_t* o
   g->d_fviews = views;
   g->d_ptab = ptab;
   g->nftables = ntables;
+  g->fguess_hit.assign((size_t)ntables, 0.0);
+  for (int t = 0; t < ntables; ++t) g->fguess_hit[(size_t)t] = tabs[t].gmode ? tabs[t].ghit : 0.0;
   g->flux0 = hv[0];
   return ok();
 }
@@ -1150,6 +1195,17 @@ mdn_status mdnorm_debug_last_launch(mdn_grid* g, int64_t out[4]) {
   out[1] = c.last_nhit;
   out[2] = mdn::walk_big_claim_threshold(g->g.n[2] > 1, g->num_sms);
   out[3] = g->slab_limit;
+  return ok();
+}
+
+mdn_status mdnorm_debug_flux_guess(mdn_grid* g, int32_t table, double out[2]) {
+  if (!g || !out) return fail(MDN_EINVAL, "NULL argument");
+  if (table < 0 || table >= g->nftables) return fail(MDN_EINVAL, "table %d outside [0, %d)", table, g->nftables);
+  std::vector<mdn::FluxView> hv(1);
+  DeviceGuard dg(g->device);
+  MDN_CUDA(cudaMemcpy(hv.data(), g->d_fviews + table, sizeof(mdn::FluxView), cudaMemcpyDeviceToHost), "view D2H");
+  out[0] = (double)hv[0].gmode;
+  out[1] = g->fguess_hit[(size_t)table];
   return ok();
 }
 

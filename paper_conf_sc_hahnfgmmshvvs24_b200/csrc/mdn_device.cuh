@@ -165,6 +165,10 @@ struct FluxView {
   const void* tab;     // ntab cell entries: int32 (global) or uint16 (shared-memory copy)
   double k_first, F_first, k_last, F_last, inv_cell;
   int n, ntab;
+  // interval guess (0: none; 1: knots near-uniform in k; 2: near-uniform in 1/k, i.e. in
+  // wavelength): i ~ floor(fma(T(x), ga, gb)) in fp32, T(x) = x or 1/x
+  float ga, gb;
+  int gmode;
 };
 
 template <typename TabT>
@@ -195,9 +199,33 @@ __device__ __forceinline__ double flux_general(const FluxView& f, double x) {
   return flux_interp(x, f.ka[lo], f.kb[lo], f.kn[lo + 1]);
 }
 
+// Guessed interval (set_flux picks the mode when the guess is right for most of the k range):
+// the guess is only a candidate -- it is accepted iff kappa_i <= x < kappa_{i+1} (and x >
+// kappa_0), which identifies the same unique interval the search finds (knots strictly
+// increase), so the value is the search path's bit for bit.  It replaces the cell-table load
+// and its dependent record loads with three independent loads (ka_i, kb_i, kappa_{i+1}).
+__device__ __forceinline__ bool flux_guess(const FluxView& f, double x, double& F) {
+  const float xf = __double2float_rn(x);
+  float u = xf;
+  if (f.gmode == 2) asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(u) : "f"(xf));
+  int i = __float2int_rd(__fmaf_rn(u, f.ga, f.gb));
+  i = min(max(i, 0), f.n - 2);
+  const double2 a = f.ka[i], b = f.kb[i];
+  const double kn1 = f.ka[i + 1].x;
+  if (a.x <= x && x < kn1 && x > f.k_first) {
+    F = flux_interp(x, a, b, kn1);
+    return true;
+  }
+  return false;
+}
+
 template <typename TabT = int>
 __device__ __forceinline__ double flux_at(const FluxView& f, double x) {
   constexpr unsigned flag = sizeof(TabT) == 2 ? kFluxDense16 : kFluxDense32;
+  if (f.gmode != 0) {
+    double F;
+    if (flux_guess(f, x, F)) return F;
+  }
   const int c = __double2int_rd(dmul(dsub(x, f.k_first), f.inv_cell));
   const unsigned e = (unsigned)c < (unsigned)f.ntab ? tab_entry<TabT>(f, c) : flag;
   if (e & flag) return flux_general(f, x);

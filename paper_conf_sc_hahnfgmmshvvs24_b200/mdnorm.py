@@ -377,6 +377,13 @@ def mdnorm_debug_last_launch(g: Grid) -> dict:
     return dict(zip(("slabs", "hitters", "big_claim_threshold", "slab_limit"), (int(x) for x in out)))
 
 
+def mdnorm_debug_flux_guess(g: Grid, table: int = 0) -> dict:
+    """{mode, hit}: the flux interval guess chosen for a table (0 none, 1 uniform in k, 2 in 1/k)."""
+    out = np.zeros(2, np.float64)
+    check(load().mdnorm_debug_flux_guess(g.handle, int(table), out.ctypes.data), "mdnorm_debug_flux_guess")
+    return {"mode": int(out[0]), "hit": float(out[1])}
+
+
 def binmd_box_bounds(g: Grid, events, box_events=1024, bounds=None, stream=None):
     """MDBox extents (NEXT #4) of packed float4 CUDA events: a CUDA float32 tensor [nboxes, 6]
     (allocated if None) of (min Qx, Qy, Qz, max Qx, Qy, Qz) per box of box_events events."""

@@ -18,7 +18,7 @@ def lib():
 
 def test_header_symbols_exported(lib):
     names = _native.header_functions()
-    assert len(names) == 30
+    assert len(names) == 31
     for n in names:
         assert hasattr(lib, n), f"{n} declared in include/mdnorm.h but not exported"
         assert n in _native.SIGNATURES, f"{n} missing from the Python binding"
