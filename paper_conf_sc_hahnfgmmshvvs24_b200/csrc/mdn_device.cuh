@@ -204,14 +204,28 @@ __device__ __forceinline__ double flux_general(const FluxView& f, double x) {
 // kappa_0), which identifies the same unique interval the search finds (knots strictly
 // increase), so the value is the search path's bit for bit.  It replaces the cell-table load
 // and its dependent record loads with three independent loads (ka_i, kb_i, kappa_{i+1}).
+template <typename TabT>
 __device__ __forceinline__ bool flux_guess(const FluxView& f, double x, double& F) {
   const float xf = __double2float_rn(x);
   float u = xf;
   if (f.gmode == 2) asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(u) : "f"(xf));
   int i = __float2int_rd(__fmaf_rn(u, f.ga, f.gb));
   i = min(max(i, 0), f.n - 2);
-  const double2 a = f.ka[i], b = f.kb[i];
-  const double kn1 = f.ka[i + 1].x;
+  double2 a, b;
+  double kn1;
+  if constexpr (sizeof(TabT) == 2) {
+    // shared-memory records: the three loads are issued together, before the acceptance test
+    // (left to itself the compiler sinks the kb load behind it: one more dependent round trip)
+    const unsigned sa = (unsigned)__cvta_generic_to_shared(f.ka + i);
+    const unsigned sb = (unsigned)__cvta_generic_to_shared(f.kb + i);
+    asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(a.x), "=d"(a.y) : "r"(sa));
+    asm volatile("ld.shared.f64 %0, [%1+16];" : "=d"(kn1) : "r"(sa));
+    asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(b.x), "=d"(b.y) : "r"(sb));
+  } else {
+    a = f.ka[i];
+    b = f.kb[i];
+    kn1 = f.ka[i + 1].x;
+  }
   if (a.x <= x && x < kn1 && x > f.k_first) {
     F = flux_interp(x, a, b, kn1);
     return true;
@@ -224,7 +238,7 @@ __device__ __forceinline__ double flux_at(const FluxView& f, double x) {
   constexpr unsigned flag = sizeof(TabT) == 2 ? kFluxDense16 : kFluxDense32;
   if (f.gmode != 0) {
     double F;
-    if (flux_guess(f, x, F)) return F;
+    if (flux_guess<TabT>(f, x, F)) return F;
   }
   const int c = __double2int_rd(dmul(dsub(x, f.k_first), f.inv_cell));
   const unsigned e = (unsigned)c < (unsigned)f.ntab ? tab_entry<TabT>(f, c) : flag;
