@@ -239,22 +239,38 @@ __device__ __forceinline__ int class_axis0(const BinTables& T, int c, float q0, 
   return axis_decide(axis_t(x, q0, q1, q2), fmaf(T.sCB[c].x, qm, T.bd[0]), T.bM[0]);
 }
 
-// Bin of member m of class c whose first axis gave i0 (>= 0, or -2 undecided), or -1: the
-// remaining two axes in fp32 inside their bands (d1, d2: the class's, for this event), and the
-// exact fp64 formula for each axis left undecided.
-__device__ __forceinline__ int member_bin(const BinParams& p, const BinTables& T, int m, float q0, float q1,
-                                          float q2, int i0, float d1, float d2) {
-  const float4 f1 = T.sMF[2 * m], f2 = T.sMF[2 * m + 1];
-  const float t1 = fmaf(f1.z, q2, fmaf(f1.y, q1, fmaf(f1.x, q0, -f1.w)));
-  const float t2 = fmaf(f2.z, q2, fmaf(f2.y, q1, fmaf(f2.x, q0, -f2.w)));
-  int i1 = axis_decide(t1, d1, T.bM[1]);
-  int i2 = axis_decide(t2, d2, T.bM[2]);
-  if (i1 == -1 || i2 == -1) return -1;
-  const double* N = T.sN + 9 * m;
+// The remaining two axes of one member after the fp32 pass could not decide them (rare; kept
+// out of line): axis_decide's verdicts from the directed bounds (rl, rh), the exact fp64 formula
+// for each axis left undecided (and for the first axis when i0 = -2).
+__device__ __forceinline__ int member_bin_slow(const BinParams& p, const double* N, float q0, float q1, float q2,
+                                            int i0, float rl1, float rh1, float rl2, float rh2) {
+  int i1 = (rl1 == rh1 && rl1 >= kMagic) ? __float_as_int(rl1) - __float_as_int(kMagic) : -2;
+  int i2 = (rl2 == rh2 && rl2 >= kMagic) ? __float_as_int(rl2) - __float_as_int(kMagic) : -2;
   if (i0 == -2 && (i0 = axis_exact(p.g, N, p.ord[0], q0, q1, q2)) < 0) return -1;
   if (i1 == -2 && (i1 = axis_exact(p.g, N, p.ord[1], q0, q1, q2)) < 0) return -1;
   if (i2 == -2 && (i2 = axis_exact(p.g, N, p.ord[2], q0, q1, q2)) < 0) return -1;
   return i0 * p.st[0] + i1 * p.st[1] + i2 * p.st[2];
+}
+
+// Bin of member m of class c whose first axis gave i0 (>= 0, or -2 undecided), or -1: the
+// remaining two axes in fp32 inside their bands (d1, d2: the class's, for this event), and the
+// exact fp64 formula for each axis left undecided -- axis_decide's rules for both axes at once,
+// with one branch on the common outcome (both decided, first axis decided) and the rest out of line.
+__device__ __forceinline__ int member_bin(const BinParams& p, const BinTables& T, int m, float q0, float q1,
+                                          float q2, int i0, float d1, float d2, float M1, float M2, int st0,
+                                          int st1, int st2) {
+  const float4 f1 = T.sMF[2 * m], f2 = T.sMF[2 * m + 1];
+  const float t1 = fmaf(f1.z, q2, fmaf(f1.y, q1, fmaf(f1.x, q0, -f1.w)));
+  const float t2 = fmaf(f2.z, q2, fmaf(f2.y, q1, fmaf(f2.x, q0, -f2.w)));
+  const float rl1 = __fadd_rd(__fsub_rd(t1, d1), kMagic), rh1 = __fadd_rd(__fadd_ru(t1, d1), kMagic);
+  const float rl2 = __fadd_rd(__fsub_rd(t2, d2), kMagic), rh2 = __fadd_rd(__fadd_ru(t2, d2), kMagic);
+  // axis_decide's "outside" on either axis
+  if (rh1 < kMagic || rl1 >= M1 || rh2 < kMagic || rl2 >= M2) return -1;
+  // both decided (not outside, equal floors: rl >= kMagic follows from rh >= kMagic)
+  if (rl1 == rh1 && rl2 == rh2 && i0 >= 0)
+    return i0 * st0 + (__float_as_int(rl1) - __float_as_int(kMagic)) * st1 +
+           (__float_as_int(rl2) - __float_as_int(kMagic)) * st2;
+  return member_bin_slow(p, T.sN + 9 * m, q0, q1, q2, i0, rl1, rh1, rl2, rh2);
 }
 
 // The class test of one event for kNC classes held in registers (kNC = 0: ncls classes read from
@@ -304,6 +320,8 @@ __device__ __forceinline__ unsigned drain_entry(const BinParams& p, const BinTab
   using PT = priv_t<kPriv>;
   unsigned inside = 0;
   const float qm = fmaxf(fabsf(ev.y), fmaxf(fabsf(ev.z), fabsf(ev.w)));
+  const float M1 = T.bM[1], M2 = T.bM[2];
+  const int st0 = p.st[0], st1 = p.st[1], st2 = p.st[2];
   // bit c < 31: class c passed; bit 31: some class >= 31 passed (each is re-tested below)
   int c = -1, cend = 0;
   for (;;) {
@@ -322,7 +340,7 @@ __device__ __forceinline__ unsigned drain_entry(const BinParams& p, const BinTab
     const int j1 = T.sCls[c + 1];
 #pragma unroll 2
     for (int j = T.sCls[c]; j < j1; ++j) {
-      const int b = member_bin(p, T, T.sMem[j], ev.y, ev.z, ev.w, i0, d1, d2);
+      const int b = member_bin(p, T, T.sMem[j], ev.y, ev.z, ev.w, i0, d1, d2, M1, M2, st0, st1, st2);
       if (b < 0) continue;
       if constexpr (kPriv != 0) hist_add<PT>(hb, he, b, (PT)ev.x, (PT)e2, has_err);
       else hist_add(p.binmd, p.err2, b, (double)ev.x, (double)e2, has_err);
@@ -527,7 +545,9 @@ debug_bins_kernel(const __grid_constant__ BinParams p, const __grid_constant__ M
     if (fabsf(axis_t(x, q0, q1, q2)) < fmaf(x.c, qm, x.d)) {
       const int i0 = class_axis0(T, c, q0, q1, q2, qm);
       const float4 cb = T.sCB[c];
-      if (i0 != -1) b = member_bin(p, T, m, q0, q1, q2, i0, fmaf(cb.y, qm, T.bd[1]), fmaf(cb.z, qm, T.bd[2]));
+      if (i0 != -1)
+        b = member_bin(p, T, m, q0, q1, q2, i0, fmaf(cb.y, qm, T.bd[1]), fmaf(cb.z, qm, T.bd[2]), T.bM[1], T.bM[2],
+                       p.st[0], p.st[1], p.st[2]);
     }
     bins[t] = b;
   }
