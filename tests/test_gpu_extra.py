@@ -303,3 +303,56 @@ def test_divide_on_bin_shards(mdn):
     with pytest.raises(ValueError):
         mdn.mdn_divide(packed[:4].cpu(), packed[:4].cpu())
     g.close()
+
+
+def _nccl_world1_worker(port, q):
+    """The X1 collectives over the NCCL backend itself (world size 1: this environment has one
+    GPU per call, and NCCL refuses two ranks on one device): reduce, all_reduce and
+    reduce_scatter_tensor on the library's own [norm | binmd | err2] device buffer."""
+    import torch
+    import torch.distributed as dist
+    sys.path.insert(0, ROOT)
+    import paper_conf_sc_hahnfgmmshvvs24_b200 as m
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    torch.cuda.set_device(0)
+    dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+    assert dist.get_backend() == "nccl"
+    wl = synth.make_workload("corelli", events_per_run=200_000)
+    ev = synth.events_for_run(wl, 0)
+    ev8 = np.zeros((len(ev), 8), np.float32)
+    ev8[:, 0] = ev[:, 0]
+    ev8[:, 1] = 0.5 * ev[:, 0] + 0.25
+    ev8[:, 5:8] = ev[:, 1:4]
+    g = m.mdnorm_create_grid(0, wl.lo, wl.hi, [61, 47, 1], wl.W)
+    m.mdnorm_set_instrument(g, wl.pix_dir, wl.solid)
+    m.mdnorm_set_flux(g, wl.flux_k, wl.flux_F)
+    m.mdnorm_accumulate(g, wl.UB, wl.R[0], wl.ops, wl.k_min, wl.k_max, 1.0, pix_stride=11)
+    m.binmd_accumulate_err(g, wl.UB, wl.ops, torch.from_numpy(ev8).cuda(), col_w=0, col_e=1, col_q=5)
+    packed = m.packed_histograms(g)
+    n = g.nbins_total
+    before = packed.clone()
+    m.reduce_packed(packed, dst=0, nbins=n)          # NCCL reduce of [norm | binmd]
+    m.reduce_packed(packed, dst=None, nbins=n, with_err=True)  # NCCL all_reduce of all three parts
+    ns, bs, es, (b0, b1) = m.reduce_scatter_packed(packed, nbins=n, with_err=True)  # NCCL reduce_scatter
+    torch.cuda.synchronize()
+    q.put((before.cpu().numpy(), packed.cpu().numpy(), ns.cpu().numpy(), bs.cpu().numpy(), es.cpu().numpy(),
+           b0, b1, n))
+    g.close()
+    dist.destroy_process_group()
+
+
+def test_nccl_backend_collectives_world1(mdn):
+    """dist.py's collectives executed by NCCL on the library's device buffer (a one-rank sum is
+    the identity, so every part must come back bit-identical)."""
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    p = ctx.Process(target=_nccl_world1_worker, args=(_free_port(), q))
+    p.start()
+    before, after, ns, bs, es, b0, b1, n = q.get(timeout=600)
+    p.join(timeout=120)
+    assert p.exitcode == 0
+    assert np.array_equal(before, after)
+    assert (b0, b1) == (0, n)
+    assert np.array_equal(ns, before[:n]) and np.array_equal(bs, before[n:2 * n]) and np.array_equal(es, before[2 * n:])
+    assert before[:n].any() and before[n:2 * n].any() and before[2 * n:].any()
