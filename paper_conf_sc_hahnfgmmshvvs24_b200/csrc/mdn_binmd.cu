@@ -497,8 +497,10 @@ binmd_kernel(const __grid_constant__ BinParams p, const __grid_constant__ MatBlo
     priv_zero(hb, p.g.nbins);
     if (p.col_e >= 0) priv_zero(he, p.g.nbins);
   }
-  // the divide after BinMD (launch_cross_section, programmatic dependent launch) may launch now;
-  // it waits for this grid to complete before reading either histogram
+  // a kernel launched after BinMD with programmatic dependent launch (the MDNorm cull in the
+  // bench step order, or the divide) may start its CTAs on the SMs this grid's CTAs leave; it
+  // executes griddepcontrol.wait before anything that depends on this grid (the divide before
+  // reading the histograms, the cull at its very end) -- this trigger only allows the early start
   asm volatile("griddepcontrol.launch_dependents;");
   load_tables(p.tables, T);
   const int w = threadIdx.x >> 5;
