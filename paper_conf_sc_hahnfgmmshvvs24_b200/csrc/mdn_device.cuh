@@ -169,6 +169,9 @@ struct FluxView {
   // wavelength): i ~ floor(fma(T(x), ga, gb)) in fp32, T(x) = x or 1/x
   float ga, gb;
   int gmode;
+  // shared-window addresses of ka and kb (shared-memory copy only): the look-up adds 16 i instead
+  // of converting a generic pointer on every call
+  unsigned ska, skb;
 };
 
 template <typename TabT>
@@ -216,8 +219,8 @@ __device__ __forceinline__ bool flux_guess(const FluxView& f, double x, double& 
   if constexpr (sizeof(TabT) == 2) {
     // shared-memory records: the three loads are issued together, before the acceptance test
     // (left to itself the compiler sinks the kb load behind it: one more dependent round trip)
-    const unsigned sa = (unsigned)__cvta_generic_to_shared(f.ka + i);
-    const unsigned sb = (unsigned)__cvta_generic_to_shared(f.kb + i);
+    const unsigned sa = f.ska + 16u * (unsigned)i;
+    const unsigned sb = f.skb + 16u * (unsigned)i;
     asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(a.x), "=d"(a.y) : "r"(sa));
     asm volatile("ld.shared.f64 %0, [%1+16];" : "=d"(kn1) : "r"(sa));
     asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(b.x), "=d"(b.y) : "r"(sb));

@@ -27,8 +27,14 @@ using namespace common;
 // One persistent walk CTA per SM (the shared-memory flux table takes up to 196 KB): 1024
 // threads for 2-D slices (64 registers: measured 1024 > 896 > 768 on the CORELLI slab), 768 for
 // 3-D grids (the unrolled walk needs more registers).
-constexpr int kWalkThreads2D = 1024;
-constexpr int kWalkThreads3D = 768;
+#ifndef MDN_WALK_THREADS_2D
+#define MDN_WALK_THREADS_2D 1024
+#endif
+#ifndef MDN_WALK_THREADS_3D
+#define MDN_WALK_THREADS_3D 768
+#endif
+constexpr int kWalkThreads2D = MDN_WALK_THREADS_2D;
+constexpr int kWalkThreads3D = MDN_WALK_THREADS_3D;
 // walk warps claim hitters kWalkChunk at a time (near the end of a launch) into a per-warp ring
 constexpr int kWalkChunk = 8;
 // the last kWalkSplitTail hitters per warp are cut into kWalkSplit x more pieces (measured: 4 > 8
@@ -435,6 +441,8 @@ __device__ __forceinline__ FluxView stage_flux(const MdnParams& p, double2* sKa,
     // the rare general path bisects the global knots (fx.kn)
     fx.ka = sKa;
     fx.kb = sKb;
+    fx.ska = (unsigned)__cvta_generic_to_shared(sKa);
+    fx.skb = (unsigned)__cvta_generic_to_shared(sKb);
   }
   return fx;
 }
