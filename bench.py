@@ -580,6 +580,15 @@ def run_ours(args, rank, world, local_rank):
                                "traffic": traffic.get("binmd_kernel"), "ms": ph_ms["binmd"],
                                "bytes_per_launch": bm_bytes,
                                "peak_source": f"{peaks_src}: MEASURED_PEAKS.json hbm_gbs"}
+    if aroof:
+        # the stream and the in-grid reductions do not overlap (profiles/r02_binmd_ablation.md):
+        # serial floor = bytes at the measured copy bandwidth + reductions at the measured roof
+        reds = stats["event_op_inside"]
+        floor_s = bm_bytes / (hbm * 1e9) + reds / aroof
+        kernels["binmd_kernel"]["serial_floor"] = {
+            "bound": "hbm+atomic", "stream_us": bm_bytes / (hbm * 1e9) * 1e6, "reductions": reds,
+            "reductions_us": reds / aroof * 1e6, "floor_us": floor_s * 1e6, "frac": floor_s / tb,
+            "source": "profiles/r02_binmd_ablation.md (decisions hide under the stream; the reductions add to it)"}
     tx = ph_ms["xs"] / 1e3
     if rank == 0 and tx > 0:
         xs_bytes = 24 * g.nbins_total
@@ -593,7 +602,7 @@ def run_ours(args, rank, world, local_rank):
             "ncu_walk": walk, "ncu_cull": nb["kernels"].get("mdnorm_cull_kernel", {}), "source": nb.get("source")}
     if nb["kernels"].get("binmd_kernel"):
         kernels["binmd_kernel"]["binding"] = {
-            "resource": "latency and per-SM imbalance of the in-grid (event, op) decisions and their reductions",
+            "resource": "the event stream plus its in-grid fp64 L2 reductions, serialised (profiles/r02_binmd_ablation.md)",
             "ncu": nb["kernels"]["binmd_kernel"], "source": nb.get("source")}
     dom = max(("mdnorm", "binmd_kernel"), key=lambda k: kernels[k]["ms"])
     roof = {k: kernels[dom][k] for k in ("bound", "achieved", "peak", "unit", "frac", "traffic")}
