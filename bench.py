@@ -360,6 +360,29 @@ class Case:
             del ev_d
             self.ev_host = None
             self.event_note = "10^8 events per run = ten copies of one seeded Morton-ordered 10^7-event draw"
+        elif name == "stress":
+            # configs[4]: one TOPAZ-shaped run on the 500^3 grid (1 GB per histogram part: every
+            # reduction goes to HBM), nops ops (default 48), 10^9 events for the whole job, strong-
+            # scaled: pixels interleaved by rank, events in contiguous blocks, ONE reduce_scatter
+            # (the grid is too large to gather) and a divide of each rank's bin block
+            wl = synth.make_workload("stress", nops=nops or 48)
+            from paper_conf_sc_hahnfgmmshvvs24_b200 import plan_shards
+            total_ev = 1_000_000_000
+            plan = plan_shards(world, rank, 1, wl.npix, total_ev)
+            self.runs = [0]
+            self.pix = (plan.pix_begin, plan.pix_stride)
+            self.scaling = "strong"
+            b, e = plan.event_ranges[0]
+            ev = synth.events_for_run(wl, 0, n=10_000_000)
+            ev_d = torch.from_numpy(ev).to(dev)
+            self.ev_dev = torch.empty((e - b, 4), dtype=torch.float32, device=dev)
+            for o in range(0, e - b, ev_d.shape[0]):  # copies of one Morton-ordered 10^7-event draw
+                k = min(ev_d.shape[0], e - b - o)
+                self.ev_dev[o:o + k] = ev_d[:k]
+            del ev_d
+            self.ev_host = None
+            self.event_note = (f"10^9 events for the job ({e - b} on this rank) = copies of one seeded "
+                               "Morton-ordered 10^7-event draw")
         else:
             raise ValueError(name)
         self.wl = wl
@@ -375,6 +398,11 @@ class Case:
         self.traj_total = (wl.nruns if name == "multirun" else world) * wl.npix * wl.nops
         self.events_total = self.events_rank * (1 if name == "multirun" else world) if name != "multirun" \
             else wl.nruns * self.ev_dev.shape[0]
+        if name == "stress":
+            pb, ps = self.pix
+            self.traj_rank = len(range(pb, wl.npix, ps)) * wl.nops
+            self.traj_total = wl.npix * wl.nops
+            self.events_total = 1_000_000_000
 
     def step(self, ph=None, events=None):
         """mdnorm_reset + BinMD of this rank's runs' events + MDNorm of the runs (+ one reduce of
@@ -390,7 +418,10 @@ class Case:
                 m.binmd_accumulate(g, wl.UB, wl.ops, self.ev_dev if events is None else events)
 
         def mdnorm():
-            if len(self.runs) == 1:
+            if self.name == "stress":
+                m.mdnorm_accumulate(g, wl.UB, wl.R[0], wl.ops, wl.k_min, wl.k_max, float(wl.charge[0]),
+                                    pix_begin=self.pix[0], pix_stride=self.pix[1])
+            elif len(self.runs) == 1:
                 r = self.runs[0]
                 m.mdnorm_accumulate(g, wl.UB, wl.R[r], wl.ops, wl.k_min, wl.k_max, float(wl.charge[r]))
             else:
@@ -404,6 +435,13 @@ class Case:
         rec(1)
         second()
         rec(2)
+        if self.name == "stress" and self.world > 1:
+            # the 2 GB [norm | binmd] is reduce-scattered; every rank divides its own bin block
+            norm, bm, _ = m.reduce_scatter_packed(self.packed, nbins=g.nbins_total)
+            rec(3)
+            m.mdn_divide(norm, bm, xs=self.xs_dev[: norm.numel()])
+            rec(4)
+            return
         if self.world > 1:
             m.reduce_packed(self.packed, dst=0, nbins=g.nbins_total)
         rec(3)
@@ -415,15 +453,21 @@ class Case:
         wl = self.wl
         d = {"workload": {"corelli": "corelli (BASELINE.json configs[1])",
                           "multirun": "corelli multi-run rotation scan (BASELINE.json configs[3])",
-                          "topaz": f"topaz, {wl.nops} ops (BASELINE.json configs[2])"}[self.name],
-             "pixels": wl.npix, "ops": wl.nops, "runs_total": wl.nruns if self.name == "multirun" else self.world,
+                          "topaz": f"topaz, {wl.nops} ops (BASELINE.json configs[2])",
+                          "stress": f"stress: 500^3 grid, {wl.nops} ops, 10^9 events (BASELINE.json configs[4])"
+                          }[self.name],
+             "pixels": wl.npix, "ops": wl.nops,
+             "runs_total": wl.nruns if self.name == "multirun" else (1 if self.name == "stress" else self.world),
              "runs_per_gpu": len(self.runs), "trajectories_per_gpu": self.traj_rank,
              "events_per_gpu": self.events_rank, "events": self.event_note,
              "grid": [int(x) for x in wl.nbins],
              "grid_extent": [[float(a), float(b)] for a, b in zip(wl.lo, wl.hi)],
              "event_order": "coarse-Q Morton (MDBox/SaveMD order)", "acc": "fp64",
              "l2": "flushed between timed steps (256 MiB device write)"}
-        if self.world > 1:
+        if self.world > 1 and self.name == "stress":
+            d["parallelism"] = (f"dp{self.world}: pixels interleaved by rank, events in contiguous blocks; "
+                                "one NCCL reduce_scatter of [norm | binmd], each rank divides its bin block")
+        elif self.world > 1:
             d["parallelism"] = (f"dp{self.world}: " + ("rank r = run r" if self.scaling == "weak"
                                                         else "contiguous run blocks per rank")
                                 + "; one NCCL reduce of [norm | binmd] to rank 0")
@@ -688,10 +732,10 @@ def main():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--config", choices=["corelli", "multirun", "topaz"], default="corelli",
+    ap.add_argument("--config", choices=["corelli", "multirun", "topaz", "stress"], default="corelli",
                     help="headline workload (default: BASELINE.json configs[1])")
-    ap.add_argument("--nops", type=int, default=None, help="symmetry ops of the topaz config (default 48)")
-    ap.add_argument("--extra-configs", default="multirun,topaz",
+    ap.add_argument("--nops", type=int, default=None, help="symmetry ops of the topaz / stress config (default 48)")
+    ap.add_argument("--extra-configs", default="multirun,topaz,stress",
                     help="other BASELINE configs timed in the same run and reported under 'configs' ('' = none)")
     ap.add_argument("--extra-weak", action="store_true", help="also time the topaz extra at N > 1")
     ap.add_argument("--no-cpu-baseline", action="store_true")
