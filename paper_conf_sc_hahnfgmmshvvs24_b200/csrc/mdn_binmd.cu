@@ -71,7 +71,9 @@ struct alignas(16) BinTables {
   int sCid[kMaxMats];        // class of matrix m
   int sCls[kMaxMats + 1];    // members of class c: sMem[sCls[c] .. sCls[c+1])
   int sMem[kMaxMats];
-  float bd[3], bn[3], bM[3]; // per test-order axis: band offset d, n, kMagic + n (fast path)
+  float bd[3], bn[3], bM[3]; // per test-order axis: band offset d, n, kMagic + n (fast path); bM[0]
+                             // is kMagic + w1 (the end of the axis-0 window)
+  float bL0;                 // kMagic + w0 (the start of the axis-0 window)
   int ncls;
   // plan scratch (not copied to the event kernel)
   AxisF sMA[kMaxMats * 2];   // member constants of test-order axes 1 and 2 (by matrix)
@@ -85,13 +87,15 @@ __device__ __forceinline__ AxisF make_axis(const BinParams& p, const double* N, 
   const double* row = N + 3 * a;
   const double s = p.g.s[a], lo = p.g.lo[a], n = (double)p.g.n[a];
   const double sum = fabs(row[0]) + fabs(row[1]) + fabs(row[2]);
+  // the class test (fold, axis 0) is centred on the launch's window [w0, w1) of the axis
+  const double wc = 0.5 * ((double)p.w0 + (double)p.w1), wh = 0.5 * ((double)p.w1 - (double)p.w0);
   AxisF x;
   x.a0 = (float)(row[0] * s);
   x.a1 = (float)(row[1] * s);
   x.a2 = (float)(row[2] * s);
-  x.b = (float)(fold ? lo * s + 0.5 * n : lo * s);
+  x.b = (float)(fold ? lo * s + wc : lo * s);
   x.c = (float)(1e-6 * s * sum);
-  x.d = (float)(1e-6 * (fabs(lo * s) + n + 1.0) + (fold ? 0.5 * n : 0.0));
+  x.d = (float)(1e-6 * (fabs(lo * s) + n + 1.0) + (fold ? wh : 0.0));
   x.n = (float)n;
   x.pad = 0.f;
   return x;
@@ -136,8 +140,9 @@ __device__ void build_tables(const BinParams& p, const MatBlock& mb, BinTables& 
     // axes of 2^21 bins or more take the exact path always (the fast floor needs |t| < 2^22)
     T.bd[k] = n < 2097152.0 ? (float)(1e-6 * (fabs(p.g.lo[a] * p.g.s[a]) + n + 1.0)) : 1e30f;
     T.bn[k] = (float)n;
-    T.bM[k] = kMagic + (float)n;
+    T.bM[k] = kMagic + (float)(k == 0 ? p.w1 : n);
   }
+  if (threadIdx.x == 0) T.bL0 = kMagic + (float)p.w0;
   __syncthreads();
   // classes: the class-test row (a0, a1, a2) decides (b and d are per axis; the band slope c is
   // taken as the class maximum below).  rep(m) = first r <= m with the same row.
@@ -216,11 +221,11 @@ __device__ void build_tables(const BinParams& p, const MatBlock& mb, BinTables& 
 // lo = RD(t - d) <= t64 <= hi = RU(t + d): floor(lo) and floor(hi) come from one directed add of
 // kMagic each; equal floors inside [0, n) decide the bin, hi < 0 or lo >= n decide "outside",
 // anything else is left to the exact fp64 formula (-2).
-__device__ __forceinline__ int axis_decide(float t, float d, float Mn) {
+__device__ __forceinline__ int axis_decide(float t, float d, float Mn, float M0 = kMagic) {
   const float rl = __fadd_rd(__fsub_rd(t, d), kMagic);
   const float rh = __fadd_rd(__fadd_ru(t, d), kMagic);
-  if (rh < kMagic || rl >= Mn) return -1;
-  if (rl == rh && rl >= kMagic) return __float_as_int(rl) - __float_as_int(kMagic);
+  if (rh < M0 || rl >= Mn) return -1;
+  if (rl == rh && rl >= M0) return __float_as_int(rl) - __float_as_int(kMagic);
   return -2;
 }
 
@@ -236,7 +241,7 @@ __device__ __forceinline__ int axis_exact(const GridC& g, const double* N, int a
 // First test-order axis of a queued (event, class): -1 outside, -2 undecided, else the bin.
 __device__ __forceinline__ int class_axis0(const BinTables& T, int c, float q0, float q1, float q2, float qm) {
   const AxisF x = T.sC0[c];
-  return axis_decide(axis_t(x, q0, q1, q2), fmaf(T.sCB[c].x, qm, T.bd[0]), T.bM[0]);
+  return axis_decide(axis_t(x, q0, q1, q2), fmaf(T.sCB[c].x, qm, T.bd[0]), T.bM[0], T.bL0);
 }
 
 // The remaining two axes of one member after the fp32 pass could not decide them (rare; kept
@@ -246,7 +251,7 @@ __device__ __forceinline__ int member_bin_slow(const BinParams& p, const double*
                                             int i0, float rl1, float rh1, float rl2, float rh2) {
   int i1 = (rl1 == rh1 && rl1 >= kMagic) ? __float_as_int(rl1) - __float_as_int(kMagic) : -2;
   int i2 = (rl2 == rh2 && rl2 >= kMagic) ? __float_as_int(rl2) - __float_as_int(kMagic) : -2;
-  if (i0 == -2 && (i0 = axis_exact(p.g, N, p.ord[0], q0, q1, q2)) < 0) return -1;
+  if (i0 == -2 && ((i0 = axis_exact(p.g, N, p.ord[0], q0, q1, q2)) < p.w0 || i0 >= p.w1)) return -1;
   if (i1 == -2 && (i1 = axis_exact(p.g, N, p.ord[1], q0, q1, q2)) < 0) return -1;
   if (i2 == -2 && (i2 = axis_exact(p.g, N, p.ord[2], q0, q1, q2)) < 0) return -1;
   return i0 * p.st[0] + i1 * p.st[1] + i2 * p.st[2];

@@ -95,6 +95,8 @@ struct BinParams {
   int32_t col_e;           // error-squared column, or -1
   int32_t ord[3];          // axis test order of the fp32 fast path (fewest bins first)
   int32_t st[3];           // linear-index stride of axis ord[k] (1, n0, n0 n1)
+  int32_t w0, w1;          // bins [w0, w1) of test-order axis 0 are scattered (an L2-sized slab of a
+                           // grid larger than L2, one launch per slab); [0, n) otherwise
   int32_t acc_f32;         // privatised partial sums in fp32 (MDN_ACC_F32) instead of fp64
   int32_t priv;            // shared-memory privatised histogram: -1 auto, 0 never, 1 whenever it fits
   double* binmd;           // fp64 histogram (nbins)
