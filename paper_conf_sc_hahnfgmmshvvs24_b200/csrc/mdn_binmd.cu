@@ -422,7 +422,7 @@ __device__ __forceinline__ void binmd_loop(const BinParams& p, const MatBlock& m
     return make_float4(0.f, 0.f, 0.f, 0.f);
   };
   auto test = [&](const float4& ev, float e2, bool valid) {
-    if (kStats && valid) c_pairs += mb.nmat;
+    if (kStats && valid && p.w0 == 0) c_pairs += mb.nmat;  // once per event over the L2 slabs
     const float qm = fmaxf(fabsf(ev.y), fmaxf(fabsf(ev.z), fabsf(ev.w)));
     unsigned mask = ct(T, ev.y, ev.z, ev.w, qm);
     if (!valid) mask = 0;
