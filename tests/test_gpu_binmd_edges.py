@@ -89,3 +89,44 @@ def test_binmd_edges_privatised(mdn):
     assert mdn.mdnorm_accumulation_paths(g)[1] != "global"
     bm = mdn.packed_histograms(g).cpu().numpy()[g.nbins_total:2 * g.nbins_total]
     assert np.array_equal(bm, oracle.binmd(oracle.Grid(lo, hi, n), N, ev))
+
+
+def test_binmd_l2_slabs_boundaries(mdn):
+    """BinMD on a grid larger than L2 (binmd part 154 MB: two L2 slabs of the last axis, one
+    launch each with an axis window, DESIGN.md §4 "BinMD on grids larger than L2"): edge events
+    on every bin plane plus events whose op image sits on the slab boundary plane itself (+-3
+    fp32 ulps), unit weights -- the histogram equals the oracle's exactly (no pair dropped or
+    counted twice at the seam), and the (event, op) pair counter counts each event once."""
+    import torch
+    wl = synth.make_workload("topaz", nops=48, events_per_run=1000)
+    lo, hi, n = [-6.0, -6.0, -3.0], [6.0, 6.0, 3.0], [400, 400, 120]
+    N = oracle.binmd_matrices(wl.UB, wl.ops, wl.W)
+    rng = np.random.default_rng(33)
+    ev = edge_events(N, lo, hi, n, 300_000, rng)
+    # the seam: z plane 60 (the slab boundary for two slabs) on the op images' last axis
+    seam = edge_events(N, lo, hi, n, 200_000, rng)
+    s = rng.integers(0, len(N), seam.shape[0])
+    x = np.einsum("eij,ej->ei", N[s], seam[:, 1:].astype(np.float64))
+    x[:, 2] = lo[2] + 60 * (hi[2] - lo[2]) / n[2]
+    q = np.einsum("eij,ej->ei", np.linalg.inv(N)[s], x).astype(np.float32)
+    steps = rng.integers(-3, 4, q.shape[0])
+    for _ in range(3):
+        q[:, 2] = np.where(steps > 0, np.nextafter(q[:, 2], np.float32(np.inf)),
+                           np.where(steps < 0, np.nextafter(q[:, 2], np.float32(-np.inf)), q[:, 2]))
+        steps = steps - np.sign(steps)
+    seam[:, 1:] = q
+    ev = np.concatenate([ev, seam])
+    g = mdn.mdnorm_create_grid(0, lo, hi, n, wl.W, mdn.MDN_ACC_F64)
+    assert 8 * g.nbins_total > 120 * 2**20  # above the L2-slab threshold
+    mdn.mdnorm_stats(g, 1, read=False)
+    mdn.binmd_accumulate(g, wl.UB, wl.ops, torch.from_numpy(ev).cuda())
+    st = mdn.mdnorm_stats(g, 0)
+    torch.cuda.synchronize()
+    bm = mdn.packed_histograms(g).cpu().numpy()[g.nbins_total:2 * g.nbins_total]
+    obm = oracle.binmd(oracle.Grid(lo, hi, n), N, ev)
+    assert np.array_equal(bm, obm)
+    assert st["event_op_pairs"] == ev.shape[0] * len(N)
+    assert st["event_op_inside"] == int(obm.sum())
+    # pairs on both sides of the seam
+    z = obm.reshape(n[2], n[1], n[0]).sum(axis=(1, 2))
+    assert z[59] > 1000 and z[60] > 1000
