@@ -31,6 +31,7 @@ struct mdn_grid {
   int64_t npix = 0;
   double* d_flux = nullptr;   // every flux table: knots (+2 pads each), then interval records
   int* d_ftab = nullptr;      // cell tables of every flux table
+  uint16_t* d_ftab16 = nullptr;  // table 0's cell table as uint16 entries (the walk's shared-memory copy)
   mdn::FluxView* d_fviews = nullptr;  // one view per flux table (device)
   int32_t* d_ptab = nullptr;  // pixel -> flux table (several tables only)
   int32_t nftables = 0;
@@ -528,6 +529,7 @@ mdn_status mdnorm_destroy(mdn_grid* g) {
   cudaFree(g->d_pkr);
   cudaFree(g->d_flux);
   cudaFree(g->d_ftab);
+  cudaFree(g->d_ftab16);
   cudaFree(g->d_fviews);
   cudaFree(g->d_ptab);
   cudaFree(g->d_hit);
@@ -589,10 +591,12 @@ mdn_status mdnorm_set_instrument(mdn_grid* g, int64_t npix, const double* dir, c
   if (g->nftables > 1) {  // so does a pixel -> flux-table map: the tables must be set again
     cudaFree(g->d_flux);
     cudaFree(g->d_ftab);
+    cudaFree(g->d_ftab16);
     cudaFree(g->d_fviews);
     cudaFree(g->d_ptab);
     g->d_flux = nullptr;
     g->d_ftab = nullptr;
+    g->d_ftab16 = nullptr;
     g->d_fviews = nullptr;
     g->d_ptab = nullptr;
     g->nftables = 0;
@@ -794,6 +798,19 @@ mdn_status mdnorm_set_flux_tables(mdn_grid* g, int32_t ntables, const int64_t* o
   }
   if (e == cudaSuccess) e = cudaMemcpy(d, all.data(), sizeof(double) * all.size(), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(tab, all_tab.data(), sizeof(int) * ntb, cudaMemcpyHostToDevice);
+  // table 0's cells as the uint16 entries the walk stages into shared memory (flag bit 15), zero
+  // padded to whole 16-byte groups; only when every interval index fits 15 bits
+  uint16_t* tab16 = nullptr;
+  if (e == cudaSuccess && tabs[0].n <= (1 << 15) - 1) {
+    std::vector<uint16_t> t16((size_t)((tabs[0].ntab + 7) & ~7), 0);
+    for (int i = 0; i < tabs[0].ntab; ++i) {
+      const unsigned c = (unsigned)tabs[0].tab[(size_t)i];
+      t16[(size_t)i] = (uint16_t)((c & (mdn::kFluxDense32 - 1)) | ((c & mdn::kFluxDense32) ? mdn::kFluxDense16 : 0u));
+    }
+    e = cudaMalloc(&tab16, sizeof(uint16_t) * t16.size());
+    if (e == cudaSuccess) e = cudaMemcpy(tab16, t16.data(), sizeof(uint16_t) * t16.size(), cudaMemcpyHostToDevice);
+    hv[0].tab16 = tab16;
+  }
   if (e == cudaSuccess) e = cudaMemcpy(views, hv.data(), sizeof(mdn::FluxView) * ntables, cudaMemcpyHostToDevice);
   if (e == cudaSuccess && ptab) e = cudaMemcpy(ptab, hpt.data(), sizeof(int32_t) * npix, cudaMemcpyHostToDevice);
   if (e != cudaSuccess) {
@@ -801,11 +818,14 @@ mdn_status mdnorm_set_flux_tables(mdn_grid* g, int32_t ntables, const int64_t* o
     cudaFree(tab);
     cudaFree(views);
     cudaFree(ptab);
+    cudaFree(tab16);
     return cuda_fail(e, "set_flux");
   }
   cudaDeviceSynchronize();
   cudaFree(g->d_flux);
   cudaFree(g->d_ftab);
+  cudaFree(g->d_ftab16);
+  g->d_ftab16 = tab16;
   cudaFree(g->d_fviews);
   cudaFree(g->d_ptab);
   g->d_flux = d;

@@ -172,6 +172,9 @@ struct FluxView {
   // shared-window addresses of ka and kb (shared-memory copy only): the look-up adds 16 i instead
   // of converting a generic pointer on every call
   unsigned ska, skb;
+  // the cell table as the uint16 entries of the shared-memory copy (zero padded to a multiple of
+  // 8 entries), or nullptr when an entry does not fit 15 bits
+  const uint16_t* tab16;
 };
 
 template <typename TabT>

@@ -422,20 +422,47 @@ struct WalkQ {
 };
 
 // kFlux 1: the flux records and the uint16 cell table into shared memory, and the view the walk
-// uses (other modes: the global view).
+// uses (other modes: the global view).  Every 16-byte load of the copy is issued before the first
+// store, so the prologue costs about one L2 round trip (the cell table arrives pre-converted to
+// uint16; a per-element loop over the int32 table took a round trip per element: 3.7% of the
+// walk's stall samples on CORELLI).
+constexpr int kStageBatch = 8;  // 16-byte loads per thread in flight
 template <int kFlux>
 __device__ __forceinline__ FluxView stage_flux(const MdnParams& p, double2* sKa, uint16_t* sTab) {
   FluxView fx = p.flux;
   if (kFlux == 1) {
     double2* sKb = sKa + p.flux.n;
-    for (int i = threadIdx.x; i < p.flux.n; i += blockDim.x) {
-      sKa[i] = p.flux.ka[i];
-      sKb[i] = p.flux.kb[i];
-    }
-    const int* gtab = static_cast<const int*>(p.flux.tab);
-    for (int i = threadIdx.x; i < p.flux.ntab; i += blockDim.x) {
-      const unsigned e = (unsigned)gtab[i];
-      sTab[i] = (uint16_t)((e & (kFluxDense32 - 1)) | ((e & kFluxDense32) ? kFluxDense16 : 0u));
+    const int n = p.flux.n, nt = (p.flux.ntab + 7) >> 3;  // records, 16-byte groups of 8 cells
+    if (p.flux.tab16) {
+      // items [ka | kb | cells] of 16 bytes; a batch = kStageBatch items per thread, all loads
+      // issued before the stores (4096 knots at 1024 threads: two batches)
+      const int total = 2 * n + nt;
+      for (int base = 0; base < total; base += kStageBatch * (int)blockDim.x) {
+        uint4 v[kStageBatch];
+#pragma unroll
+        for (int j = 0; j < kStageBatch; ++j) {
+          const int i = base + threadIdx.x + j * blockDim.x;
+          if (i < n) v[j] = __ldg(reinterpret_cast<const uint4*>(p.flux.ka) + i);
+          else if (i < 2 * n) v[j] = __ldg(reinterpret_cast<const uint4*>(p.flux.kb) + (i - n));
+          else if (i < total) v[j] = __ldg(reinterpret_cast<const uint4*>(p.flux.tab16) + (i - 2 * n));
+        }
+#pragma unroll
+        for (int j = 0; j < kStageBatch; ++j) {
+          const int i = base + threadIdx.x + j * blockDim.x;
+          if (i < 2 * n) reinterpret_cast<uint4*>(sKa)[i] = v[j];  // sKb = sKa + n
+          else if (i < total) reinterpret_cast<uint4*>(sTab)[i - 2 * n] = v[j];
+        }
+      }
+    } else {
+      for (int i = threadIdx.x; i < n; i += blockDim.x) {
+        sKa[i] = p.flux.ka[i];
+        sKb[i] = p.flux.kb[i];
+      }
+      const int* gtab = static_cast<const int*>(p.flux.tab);
+      for (int i = threadIdx.x; i < p.flux.ntab; i += blockDim.x) {
+        const unsigned e = (unsigned)gtab[i];
+        sTab[i] = (uint16_t)((e & (kFluxDense32 - 1)) | ((e & kFluxDense32) ? kFluxDense16 : 0u));
+      }
     }
     fx.tab = sTab;
     // the rare general path bisects the global knots (fx.kn)
@@ -447,7 +474,7 @@ __device__ __forceinline__ FluxView stage_flux(const MdnParams& p, double2* sKa,
   return fx;
 }
 __host__ __device__ constexpr size_t flux_smem_bytes(int kFlux, int n, int ntab) {
-  return kFlux == 1 ? 2 * sizeof(double2) * (size_t)n + sizeof(uint16_t) * (size_t)((ntab + 1) & ~1) : 0;
+  return kFlux == 1 ? 2 * sizeof(double2) * (size_t)n + 16 * (size_t)((ntab + 7) >> 3) : 0;
 }
 // per warp: scan scratch (32 int) and the hitter ring (kWalkRing indices + piece counts)
 constexpr size_t kWalkWarpBytes = sizeof(int) * 32 + 2 * sizeof(unsigned) * kWalkRing;
