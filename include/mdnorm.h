@@ -122,7 +122,10 @@ mdn_status mdnorm_accumulate_runs(mdn_grid *g, const double UB[9], int32_t nruns
  * events: float[nevents * stride_floats] (host or device; device pointers are borrowed until the
  * stream reaches the work), event e has weight events[e*stride + col_w] (column 1 of the
  * paper's 8-column array) and Q_sample = events[e*stride + col_q + 0..2] (columns 6-8,
- * P:149-150).  Fast path: stride 4, col_w 0, col_q 1 (packed float4 (w, Qx, Qy, Qz)). */
+ * P:149-150).  Fast path: stride 4, col_w 0, col_q 1 (packed float4 (w, Qx, Qy, Qz)).
+ * Grids whose fp64 histogram exceeds what the L2 holds (> 120 MB) are binned from device events
+ * in L2-sized slabs of the last axis, one kernel pass each (the events are read once per slab;
+ * the result is the same); host events are binned in one pass. */
 mdn_status binmd_accumulate(mdn_grid *g, const double UB[9], int32_t nops, const double *ops,
                             int64_t nevents, const float *events, int64_t stride_floats,
                             int32_t col_w, int32_t col_q, void *stream);
