@@ -6,7 +6,7 @@
 
 MDBox extents and box-culled BinMD, a flux table that makes the interval guess miss and one that
 has no guess (cell-table search), the multi-slab cull/walk path, the per-bank flux tables, the
-error column and its divide, and the host-event staging ring.  Prints one line per path; checks
+error column and its divide, the host-event staging ring, and BinMD in L2 slabs.  Prints one line per path; checks
 only that each call returns (numbers are the tests' business).
 """
 import os
@@ -86,6 +86,19 @@ def main():
     m.mdnorm_accumulate_runs(g, wt.UB, wt.R, np.ones(len(wt.R)), wt.ops, wt.k_min, wt.k_max, pix_stride=1999)
     torch.cuda.synchronize()
     print("topaz runs", m.mdnorm_debug_last_launch(g), flush=True)
+    g.close()
+
+    # BinMD on a grid larger than L2 (154 MB: two L2 slabs of the last axis) with the error column
+    g = m.mdnorm_create_grid(0, [-6.0, -6.0, -3.0], [6.0, 6.0, 3.0], [400, 400, 120], wt.W, m.MDN_ACC_F64)
+    evt = torch.from_numpy(synth.events_for_run(wt, 0)).cuda()
+    m.binmd_accumulate(g, wt.UB, wt.ops, evt)
+    rows = torch.zeros((evt.shape[0], 8), dtype=torch.float32, device="cuda")
+    rows[:, 0] = evt[:, 0]
+    rows[:, 1] = evt[:, 0]
+    rows[:, 5:8] = evt[:, 1:4]
+    m.binmd_accumulate_err(g, wt.UB, wt.ops, rows)
+    torch.cuda.synchronize()
+    print("l2 slabs", float(m.packed_histograms(g)[g.nbins_total:2 * g.nbins_total].sum().item()), flush=True)
     g.close()
     print("sanitize_paths: done")
 
