@@ -130,3 +130,23 @@ def test_binmd_l2_slabs_boundaries(mdn):
     # pairs on both sides of the seam
     z = obm.reshape(n[2], n[1], n[0]).sum(axis=(1, 2))
     assert z[59] > 1000 and z[60] > 1000
+
+
+def test_binmd_l2_slabs_host_vs_device(mdn):
+    """On a grid above the L2-slab threshold, host events (staging ring, one pass) and device
+    events (two L2 slabs) give the same unit-weight histogram, equal to the oracle's."""
+    import torch
+    wl = synth.make_workload("topaz", nops=24, events_per_run=200_000)
+    lo, hi, n = [-6.0, -6.0, -3.0], [6.0, 6.0, 3.0], [400, 400, 120]
+    ev = synth.events_for_run(wl, 0)
+    N = oracle.binmd_matrices(wl.UB, wl.ops, wl.W)
+    out = []
+    for src in (ev, torch.from_numpy(ev).cuda()):
+        g = mdn.mdnorm_create_grid(0, lo, hi, n, wl.W, mdn.MDN_ACC_F64)
+        mdn.binmd_accumulate(g, wl.UB, wl.ops, src)
+        torch.cuda.synchronize()
+        out.append(mdn.packed_histograms(g).cpu().numpy()[g.nbins_total:2 * g.nbins_total].copy())
+        g.close()
+    obm = oracle.binmd(oracle.Grid(lo, hi, n), N, ev)
+    assert obm.sum() > 100_000
+    assert np.array_equal(out[0], obm) and np.array_equal(out[1], obm)
