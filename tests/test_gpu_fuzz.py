@@ -86,3 +86,56 @@ def test_random_config(mdn, seed):
     assert np.array_equal(norm == 0, onorm == 0), "norm zero pattern"
     assert np.all(np.abs(norm - onorm) <= 1e-12 * np.abs(onorm)), "norm values"
     assert np.array_equal(bm, obm), "binmd counts"
+
+
+@pytest.mark.parametrize("seed", range(24))
+def test_random_config_runs_banks_errors(mdn, seed):
+    """The same random configurations with the Mantid-compatible inputs (NEXT #1) and the batched
+    rotation scan: 2-4 runs through mdnorm_accumulate_runs (random angles and charges), per-pixel
+    k limits on a random half of the pixels (some empty), 2-3 per-bank flux tables on a random
+    pixel map, and 8-column events with an error-squared column through binmd_accumulate_err --
+    against Algorithm 1 on the oracle (norm 1e-12 per bin, counts and integer error sums exact)."""
+    import torch
+    wl = random_config(100 + seed)
+    rng = np.random.default_rng(5000 + seed)
+    nruns = int(rng.integers(2, 5))
+    R = np.stack([synth.rot_y(rng.uniform(0, 360)) for _ in range(nruns)])
+    charge = rng.uniform(0.5, 2.0, nruns)
+    npix = wl.npix
+    span = wl.k_max - wl.k_min
+    pk_lo = np.full(npix, wl.k_min)
+    pk_hi = np.full(npix, wl.k_max)
+    sel = rng.random(npix) < 0.5
+    pk_lo[sel] = wl.k_min + rng.uniform(-0.2, 0.6, sel.sum()) * span
+    pk_hi[sel] = pk_lo[sel] + rng.uniform(-0.1, 0.8, sel.sum()) * span  # some empty
+    ntab = int(rng.integers(2, 4))
+    tables = [(wl.flux_k, wl.flux_F * (1.0 + 0.5 * t)) for t in range(ntab)]
+    ptab = rng.integers(0, ntab, npix).astype(np.int32)
+    g = mdn.mdnorm_create_grid(0, wl.lo, wl.hi, wl.nbins, wl.W, mdn.MDN_ACC_F64)
+    mdn.mdnorm_set_instrument(g, wl.pix_dir, wl.solid)
+    mdn.mdnorm_set_flux_tables(g, tables, ptab)
+    mdn.mdnorm_set_pixel_krange(g, pk_lo, pk_hi)
+    mdn.mdnorm_accumulate_runs(g, wl.UB, R, charge, wl.ops, wl.k_min, wl.k_max)
+    ev = synth.events_for_run(dataclasses.replace(wl, k_min=float(wl.flux_k[0]), k_max=float(wl.flux_k[-1])), 0,
+                              unit_weights=True)
+    rows = np.zeros((len(ev), 8), np.float32)
+    rows[:, 0] = ev[:, 0]
+    rows[:, 1] = rng.integers(1, 5, len(ev)).astype(np.float32)  # error^2: integer sums are exact
+    rows[:, 5:8] = ev[:, 1:]
+    mdn.binmd_accumulate_err(g, wl.UB, wl.ops, torch.from_numpy(rows).cuda())
+    torch.cuda.synchronize()
+    packed = mdn.packed_histograms(g).cpu().numpy()
+    nb = g.nbins_total
+    norm, bm, e2 = packed[:nb], packed[nb:2 * nb], packed[2 * nb:3 * nb]
+    g.close()
+    og = oracle.Grid(wl.lo, wl.hi, wl.nbins)
+    M = oracle.mdnorm_matrices(R, wl.UB, wl.ops, wl.W)
+    onorm = oracle.mdnorm_tables(og, wl.pix_dir, wl.solid, tables, ptab, M, np.repeat(charge, wl.nops),
+                                 wl.k_min, wl.k_max, pix_kmin=pk_lo, pix_kmax=pk_hi)
+    N = oracle.binmd_matrices(wl.UB, wl.ops, wl.W)
+    obm = oracle.binmd(og, N, rows, stride=8, col_w=0, col_q=5)
+    oe2 = oracle.binmd_err(og, N, rows, stride=8, col_e=1, col_q=5)
+    assert np.array_equal(norm == 0, onorm == 0), "norm zero pattern"
+    assert np.all(np.abs(norm - onorm) <= 1e-12 * np.abs(onorm)), "norm values"
+    assert np.array_equal(bm, obm), "binmd counts"
+    assert np.array_equal(e2, oe2), "error-squared sums"
