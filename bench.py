@@ -12,6 +12,11 @@ when N > 1) + cross-section: Algorithm 1 for one file per GPU.  Weak s
 processes run r of a rotation scan (omega = 17 + 3r degrees, its own seeded events), so per-GPU
 work is fixed.  value = pixel-trajectories of all ranks / max-over-ranks step time.
 
+The other BASELINE configs are timed in the same run (reported under "configs"; --config makes
+one of them the headline): multirun = configs[3], the 120-run x 24-op scan strong-scaled over the
+ranks; topaz = configs[2], 200^3 grid, 48 ops, 10^8 events (weak, N = 1 only by default); stress =
+configs[4], 500^3 grid, 48 ops, 10^9 events for the job, strong-scaled with one reduce_scatter.
+
 Prints ONE JSON line on rank 0 (contract in the task statement; fields documented in DESIGN.md §6).
 """
 from __future__ import annotations
