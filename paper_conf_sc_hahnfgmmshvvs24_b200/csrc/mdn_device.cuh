@@ -359,6 +359,27 @@ __device__ __forceinline__ AxisStream axis_stream(const GridC& g, int a, double 
   return s;
 }
 
+// The starting guesses of axis_stream without its exact fix-up (within one plane of the exact
+// range at either end; the cull's piece plan only needs that).
+__device__ __forceinline__ AxisStream axis_estimate(const GridC& g, int a, double v, double kin, double kout) {
+  AxisStream s{0, 0, 1};
+  const int n = g.n[a];
+  if (v == 0.0 || n < 2) return s;
+  const double u_in = (kin * v - g.lo[a]) * g.s[a];
+  const double u_out = (kout * v - g.lo[a]) * g.s[a];
+  if (v > 0.0) {
+    const int jlo = clamp_floor(u_in + 1.0, 1, n), jhi = clamp_floor(u_out, 0, n - 1);
+    s.j = jlo;
+    s.cnt = jhi >= jlo ? jhi - jlo + 1 : 0;
+  } else {
+    const int jA = clamp_floor(u_in, 0, n - 1), jB = clamp_floor(u_out + 1.0, 1, n);
+    s.j = jA;
+    s.cnt = jA >= jB ? jA - jB + 1 : 0;
+    s.step = -1;
+  }
+  return s;
+}
+
 // One axis of the merge: reciprocal, position (j kept as an exact double so that the edge
 // lo + j * w needs no int->double conversion), remaining count, next crossing value.
 struct AxisCursor {

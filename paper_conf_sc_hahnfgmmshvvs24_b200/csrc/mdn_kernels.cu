@@ -170,9 +170,17 @@ struct CullWarp {
       // a non-finite v (only from a singular composition) contributes nothing in the oracle
       if (isfinite(v0) && isfinite(v1) && isfinite(v2) && traj_clip_r(p.g, vv, rr, klo, khi, kin, kout)) {
         hit = true;
-        const AxisStream s0 = axis_stream(p.g, 0, v0, rr[0], kin, kout);
-        const AxisStream s1 = axis_stream(p.g, 1, v1, rr[1], kin, kout);
-        const AxisStream s2 = axis_stream(p.g, 2, v2, rr[2], kin, kout);
+        // The piece plan needs only approximate crossing ranges: the walk clamps every cut to
+        // [kin, kout] and finds each piece's crossings exactly (a cut strictly inside (kin, kout)
+        // is a plane crossing, i.e. a member of L, and a clamped one is kin or kout).  2-D slices
+        // take the estimate (measured: CORELLI MDNorm -1.8%, the 120-run scan -2.8% per step);
+        // 3-D grids keep the exact ranges (their pieces end on the box faces, where an estimate
+        // off by one plane leaves a short first or last piece: TOPAZ 48 ops +1.8%), and so do
+        // the work counters.
+        const bool exact = kStats || p.g.n[2] > 1;
+        const AxisStream s0 = exact ? axis_stream(p.g, 0, v0, rr[0], kin, kout) : axis_estimate(p.g, 0, v0, kin, kout);
+        const AxisStream s1 = exact ? axis_stream(p.g, 1, v1, rr[1], kin, kout) : axis_estimate(p.g, 1, v1, kin, kout);
+        const AxisStream s2 = exact ? axis_stream(p.g, 2, v2, rr[2], kin, kout) : axis_estimate(p.g, 2, v2, kin, kout);
         const int total = s0.cnt + s1.cnt + s2.cnt;
         // piece plan: cut at crossings of the busiest axis A, ~kPieceSegs segments per piece
         const bool a1 = s1.cnt > s0.cnt;
@@ -402,8 +410,8 @@ struct WalkQ {
         const double vA = A == 0 ? v0 : (A == 1 ? v1 : v2);
         const double rA = ddiv(1.0, vA);
         const int cA = abs(h.stepG), st = h.stepG < 0 ? -1 : 1;
-        if (mypi > 0) lo_k = plane_k(p.g, A, h.jA + st * ((mypi * cA) / myP), rA);
-        if (mypi < myP - 1) hi_k = plane_k(p.g, A, h.jA + st * (((mypi + 1) * cA) / myP), rA);
+        if (mypi > 0) lo_k = fmax(h.kin, plane_k(p.g, A, h.jA + st * ((mypi * cA) / myP), rA));
+        if (mypi < myP - 1) hi_k = fmin(h.kout, plane_k(p.g, A, h.jA + st * (((mypi + 1) * cA) / myP), rA));
       }
       int nc;
       int ns;
