@@ -172,22 +172,25 @@ struct CullWarp {
         hit = true;
         // The piece plan needs only approximate crossing ranges: the walk clamps every cut to
         // [kin, kout] and finds each piece's crossings exactly (a cut strictly inside (kin, kout)
-        // is a plane crossing, i.e. a member of L, and a clamped one is kin or kout).  2-D slices
-        // take the estimate (measured: CORELLI MDNorm -1.8%, the 120-run scan -2.8% per step);
-        // 3-D grids keep the exact ranges (their pieces end on the box faces, where an estimate
-        // off by one plane leaves a short first or last piece: TOPAZ 48 ops +1.8%), and so do
-        // the work counters.
-        const bool exact = kStats || p.g.n[2] > 1;
+        // is a plane crossing, i.e. a member of L, and a clamped one is kin or kout): measured
+        // CORELLI MDNorm -1.8%, the 120-run scan -2.8% per step.  3-D grids take the exact range
+        // of the cut axis (their pieces end on the box faces, where an estimate one plane off
+        // leaves a short first or last piece: TOPAZ 48 ops +1.8% with every range estimated);
+        // the work counters keep every range exact.
+        const bool exact = kStats;
         const AxisStream s0 = exact ? axis_stream(p.g, 0, v0, rr[0], kin, kout) : axis_estimate(p.g, 0, v0, kin, kout);
         const AxisStream s1 = exact ? axis_stream(p.g, 1, v1, rr[1], kin, kout) : axis_estimate(p.g, 1, v1, kin, kout);
         const AxisStream s2 = exact ? axis_stream(p.g, 2, v2, rr[2], kin, kout) : axis_estimate(p.g, 2, v2, kin, kout);
         const int total = s0.cnt + s1.cnt + s2.cnt;
         // piece plan: cut at crossings of the busiest axis A, ~kPieceSegs segments per piece
         const bool a1 = s1.cnt > s0.cnt;
-        const AxisStream s01 = a1 ? s1 : s0;
-        const bool a2 = s2.cnt > s01.cnt;
-        const AxisStream sa = a2 ? s2 : s01;
+        const bool a2 = s2.cnt > (a1 ? s1.cnt : s0.cnt);
         const int A = a2 ? 2 : (a1 ? 1 : 0);
+        // 3-D grids: the exact range of the cut axis (an estimate one plane off at the box faces
+        // leaves short end pieces), the others estimated
+        AxisStream sa = a2 ? s2 : (a1 ? s1 : s0);
+        if (!exact && p.g.n[2] > 1)
+          sa = axis_stream(p.g, A, A == 0 ? v0 : (A == 1 ? v1 : v2), A == 0 ? rr[0] : (A == 1 ? rr[1] : rr[2]), kin, kout);
         int P = 1, G = 1;
         const int S = p.g.n[2] > 1 ? kPieceSegs3D : kPieceSegs;
         if (total + 1 > S && sa.cnt > 1) {
